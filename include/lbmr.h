@@ -1,0 +1,156 @@
+/*
+ * lbmr.h — C ABI of the B200-native multi-level grid-refinement LBM library
+ * (liblbmr.so).  One coarse time step of nonuniform grid refinement LBM in the
+ * volume-based style of Rohde et al. [25] as optimised by Mahmoud,
+ * Salehipour and Meneghin (IPDPS 2024).  Citations "P:Lnnn" are lines of
+ * /root/reference/PAPER.md with the section / equation they fall in.
+ *
+ * Conventions shared by every call
+ * --------------------------------
+ *  - Levels L = 0 (coarsest) .. levels-1.  Level L has (nx<<L, ny<<L, nz<<L)
+ *    cells; refinement ratio 2 (§II-A), acoustic scaling: level L runs
+ *    2^L substeps per coarse step (§III).
+ *  - Host arrays are C-order, z fastest: cell (x,y,z) of level L has linear
+ *    index (x*(ny<<L) + y)*(nz<<L) + z.  Velocity arrays are interleaved
+ *    [cell][3].  All host arrays are owned by the caller; the library copies
+ *    what it needs during the call and keeps no pointer.
+ *  - Cell codes in masks (uint8): 0 = not a leaf at this level (REFINED if
+ *    its children are covered, ABSENT if a coarser leaf covers it), 1 = fluid
+ *    leaf, 2..254 = boundary-condition leaf of that class id, 255 reserved.
+ *  - Device memory: the library allocates and owns all device memory
+ *    (populations, 2 buffers per level, and the block tables); freed by
+ *    lbm_grid_destroy.  Work is enqueued on the grid's stream.
+ *  - Errors: no exception crosses the ABI.  Every call returns an
+ *    lbm_status; on a non-OK status lbm_last_error() holds a thread-local
+ *    text.  A grid whose lbm_step failed is in LBM_E_STATE until destroyed.
+ *    CUDA errors of asynchronous work surface at the next synchronising call
+ *    (lbm_macroscopic, lbm_stats, lbm_synchronize).
+ */
+#ifndef LBMR_H
+#define LBMR_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  LBM_OK = 0,
+  LBM_E_INVAL = 1,       /* bad argument (NULL pointer, bad enum, bad dims)          */
+  LBM_E_TILING = 2,      /* masks do not tile the domain exactly once       */
+  LBM_E_UNBALANCED = 3,  /* two 26-adjacent leaves differ by > 1 level */
+  LBM_E_OOM = 4,         /* device or host allocation failed                          */
+  LBM_E_CUDA = 5,        /* CUDA runtime error (text in lbm_last_error)               */
+  LBM_E_COMM = 6,        /* multi-GPU exchange error                                   */
+  LBM_E_STATE = 7,       /* call not valid in the grid's current state                 */
+  LBM_E_UNSUPPORTED = 8  /* valid request this build does not implement (KBC+D3Q19)   */
+} lbm_status;
+
+typedef enum { LBM_D3Q19 = 19, LBM_D3Q27 = 27 } lbm_lattice;       /* P:L37 §II          */
+typedef enum { LBM_BGK = 0, LBM_KBC = 1 } lbm_collision;           /* Eq.3; KBC [18] (D3Q27 only) */
+typedef enum { LBM_FP32 = 0, LBM_FP64 = 1 } lbm_precision;         /* fp32 stores shifted populations f - w */
+typedef enum {
+  LBM_BC_NOSLIP = 0,    /* halfway bounce-back [27]                          */
+  LBM_BC_VELOCITY = 1,  /* moving wall / velocity inlet: bounce-back + 6 w_i rho_w e_i.u_w,
+                           rho_w = 1 (P:L264 lid, P:L280 inlet)                                */
+  LBM_BC_OUTFLOW = 2    /* missing f_i := w_i                                         */
+} lbm_bc_kind;
+
+typedef struct {
+  int32_t nx, ny, nz;       /* level-0 cells per axis (>= 1)                                 */
+  int32_t periodic[3];      /* 1 = periodic axis; non-periodic faces use face_bc             */
+  uint8_t face_bc[6];       /* BC class (2..254) of sources outside the -x,+x,-y,+y,-z,+z
+                               faces; at edges/corners VELOCITY > NOSLIP > OUTFLOW           */
+  uint8_t pad_[2];
+  int32_t lattice;          /* lbm_lattice                                                   */
+  int32_t collision;        /* lbm_collision                                                 */
+  int32_t precision;        /* lbm_precision                                                 */
+  double omega0;            /* level-0 relaxation Δt/τ; ω_L by Eq.9                 */
+  int32_t n_ranks, rank;    /* x-slab partition; (1, 0) = whole domain on this device        */
+  void* stream;             /* cudaStream_t to enqueue on; NULL = library-owned stream      */
+} lbm_grid_desc;
+
+typedef struct lbm_grid lbm_grid;
+
+typedef struct {
+  int32_t levels;
+  int32_t Q;
+  int32_t precision;
+  int32_t kernels_per_step;          /* 2^levels - 1 fused level-step launches (pipelined Alg.1) */
+  int64_t leaves[16];                /* fluid leaves per level                                   */
+  int64_t blocks[16];                /* 8^3 blocks holding >= 1 fluid leaf                        */
+  int64_t special_blocks[16];        /* blocks with a non-same-level or BC link                   */
+  int64_t special_cells[16];         /* fluid leaves with such a link                             */
+  int64_t total_blocks[16];          /* all stored blocks incl. refined/BC-only                   */
+  int64_t device_bytes;              /* device memory held by the grid                            */
+  int64_t steps_done;                /* coarse steps since the last init                          */
+} lbm_grid_info;
+
+/* Build the block-sparse multi-level grid (§V) from per-level masks.
+ * masks[L] points to (nx<<L)*(ny<<L)*(nz<<L) codes (see conventions).  Validates
+ * exact tiling (LBM_E_TILING) and strong 2:1 balance over the 26-neighbourhood
+ * (LBM_E_UNBALANCED), the first offending level/cell going to lbm_last_error.
+ * Allocates device memory; populations start at rest equilibrium (rho=1, u=0).
+ * levels in [1, 16]; KBC requires D3Q27 (LBM_E_UNSUPPORTED otherwise). */
+lbm_status lbm_grid_create(const lbm_grid_desc* desc, int32_t levels, const uint8_t* const* masks,
+                           lbm_grid** out);
+
+/* Define boundary class `bc_class` (2..254): kind and wall velocity u_wall[3]
+ * (lattice units of the level the link lives on; NULL = 0).  Takes effect at
+ * the next lbm_step.  Undefined classes used by masks/face_bc act as NOSLIP. */
+lbm_status lbm_set_bc(lbm_grid* g, int32_t bc_class, int32_t kind, const double* u_wall);
+
+/* f = f^eq(rho, u) (Eq.5) on the fluid leaves of `level`.  rho: dense
+ * level array or NULL (= 1); u: dense interleaved [cell][3] or NULL (= 0).
+ * Resets the step counter; the next lbm_step starts from this post-streaming
+ * state. */
+lbm_status lbm_init_equilibrium(lbm_grid* g, int32_t level, const double* rho, const double* u);
+
+/* f = f^eq(rho0, u0) on every fluid leaf of every level (u0 NULL = 0). */
+lbm_status lbm_init_uniform(lbm_grid* g, double rho0, const double* u0);
+
+/* Advance n_coarse coarse time steps (Algorithm 1): the fused
+ * per-level kernels {pull streaming + BC, Explosion Eq.10, Coalescence Eq.11
+ * (gather form of Accumulate), Collision Eq.3 / KBC} in the pipelined
+ * order, replayed as a CUDA graph.  Asynchronous on the grid's stream. */
+lbm_status lbm_step(lbm_grid* g, int32_t n_coarse);
+
+/* rho (Eq.6) and u (Eq.7) of level `level` into dense host arrays (rho: cells,
+ * u: cells*3 interleaved; either may be NULL).  Cells that are not fluid
+ * leaves get NaN.  Synchronises the grid's stream. */
+lbm_status lbm_macroscopic(lbm_grid* g, int32_t level, double* rho, double* u);
+
+/* Fluid leaves per level (leaves_per_level[levels], may be NULL) and total
+ * mass sum_L sum_leaves rho * 8^-L in coarse-cell volumes (may be NULL).
+ * Synchronises. */
+lbm_status lbm_stats(lbm_grid* g, int64_t* leaves_per_level, double* total_mass);
+
+/* Grid description and sizes (no device work). */
+lbm_status lbm_grid_get_info(const lbm_grid* g, lbm_grid_info* info);
+
+/* Instrumented run for measurement: advances n_coarse steps launching the
+ * same kernels without the graph, bracketing every launch with CUDA events
+ * on the grid's stream; ms_per_level[L] receives the summed device time of
+ * level L's launches and launches_per_level[L] their count (either may be
+ * NULL).  Synchronises. */
+lbm_status lbm_profile_levels(lbm_grid* g, int32_t n_coarse, double* ms_per_level,
+                              int64_t* launches_per_level);
+
+/* Block until all work enqueued on the grid's stream is done. */
+lbm_status lbm_synchronize(lbm_grid* g);
+
+/* Destroy the grid and free its device memory; NULL is a no-op. */
+void lbm_grid_destroy(lbm_grid* g);
+
+/* Thread-local text of the last non-OK status ("" if none). */
+const char* lbm_last_error(void);
+
+/* Library version string. */
+const char* lbm_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* LBMR_H */

@@ -1,0 +1,586 @@
+// capi.cpp — C ABI of liblbmr.so (include/lbmr.h) and the level scheduler.
+//
+// Scheduler (Algorithm 1, pipelined).  Level L runs 2^L substeps
+// per coarse step.  F_L^k = the fused kernel that streams substep k
+// of level L and collides substep k+1, writing C_L^{k+1} into buf[L][(k+1)%2].
+// Driving the finest level k = 1, 2, ... and, after every F_L^k with k odd,
+// running F_{L-1}^{(k+1)/2} recursively gives an order in which every read of
+// Alg.1 sees the value it sees in the recursion:
+//   same level C_L^k, Explosion C_{L-1}^{ceil(k/2)} (constant over the two fine
+//   substeps, R-A4), Coalescence C_{L+1}^{2k-1} and C_{L+1}^{2k} (the two fine
+//   post-collision states).
+// 3 levels: F2^1 F1^1 F0^1 F2^2 F2^3 F1^2 F2^4 — 2^Lmax - 1 launches per
+// coarse step, each moving 2Q values per leaf.  One coarse step is captured
+// once into a CUDA graph per parity of the step index (level-0 buffers
+// alternate) and replayed with cudaGraphLaunch.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/lbmr.h"
+#include "grid_builder.h"
+#include "kernels.h"
+#include "lattice.h"
+
+using namespace lbmr;
+
+namespace {
+
+thread_local std::string g_err;
+
+lbm_status fail(lbm_status s, const std::string& msg) {
+  g_err = msg;
+  return s;
+}
+
+#define CUDA_TRY(call)                                                                            \
+  do {                                                                                            \
+    cudaError_t e_ = (call);                                                                      \
+    if (e_ != cudaSuccess) return fail(LBM_E_CUDA, std::string(#call) + ": " + cudaGetErrorString(e_)); \
+  } while (0)
+
+struct DevLevel {
+  int32_t* blkmap = nullptr;
+  uint8_t* types = nullptr;
+  int32_t* origin = nullptr;
+  int32_t* nbr = nullptr;
+  int32_t* special_slot = nullptr;
+  uint32_t* cellinfo = nullptr;
+  void* pop[2] = {nullptr, nullptr};
+};
+
+}  // namespace
+
+struct lbm_grid {
+  lbm_grid_desc desc{};
+  int levels = 0;
+  int Q = 19;
+  int coll = 0;
+  int prec = 0;
+  size_t tsize = 4;
+  std::vector<HostLevel> host;
+  std::vector<DevLevel> dev;
+  std::vector<double> omega;
+  BCEntry bc_host[256];
+  BCEntry* bc_dev = nullptr;
+  uint8_t face_host[27];
+  uint8_t* face_dev = nullptr;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  cudaGraphExec_t graph[2] = {nullptr, nullptr};
+  bool needs_prologue = true;
+  bool init_locked = false;  // a step ran since the last init_uniform
+  bool broken = false;
+  int64_t steps = 0;
+  int64_t device_bytes = 0;
+  std::vector<void*> allocs;
+};
+
+namespace {
+
+template <typename T>
+lbm_status dev_upload(lbm_grid* g, T** dst, const std::vector<T>& src) {
+  size_t bytes = std::max<size_t>(src.size() * sizeof(T), sizeof(T));
+  void* p = nullptr;
+  if (cudaMalloc(&p, bytes) != cudaSuccess) return fail(LBM_E_OOM, "cudaMalloc failed (tables)");
+  g->allocs.push_back(p);
+  g->device_bytes += (int64_t)bytes;
+  if (!src.empty()) CUDA_TRY(cudaMemcpy(p, src.data(), src.size() * sizeof(T), cudaMemcpyHostToDevice));
+  *dst = static_cast<T*>(p);
+  return LBM_OK;
+}
+
+lbm_status dev_alloc(lbm_grid* g, void** dst, size_t bytes) {
+  bytes = std::max<size_t>(bytes, 16);
+  void* p = nullptr;
+  if (cudaMalloc(&p, bytes) != cudaSuccess) {
+    cudaGetLastError();
+    return fail(LBM_E_OOM, "cudaMalloc failed (" + std::to_string(bytes) + " bytes)");
+  }
+  g->allocs.push_back(p);
+  g->device_bytes += (int64_t)bytes;
+  *dst = p;
+  return LBM_OK;
+}
+
+double omega_level(double omega0, int L) {
+  // Eq.(9)
+  const double p = std::ldexp(1.0, L);
+  return 2.0 * omega0 / (2.0 * p + (1.0 - p) * omega0);
+}
+
+int bc_priority(int kind) { return kind == LBM_BC_VELOCITY ? 3 : kind == LBM_BC_NOSLIP ? 2 : 1; }
+
+// face class per outside pattern (ox,oy,oz) in {-1,0,1}^3: VELOCITY > NOSLIP >
+// OUTFLOW, ties to the first face in the order -x,+x,-y,+y,-z,+z (R-A11).
+void compute_face_classes(lbm_grid* g) {
+  for (int i = 0; i < 27; ++i) {
+    int o[3] = {i % 3 - 1, (i / 3) % 3 - 1, i / 9 - 1};
+    int best = g->desc.face_bc[0], bp = -1;
+    for (int a = 0; a < 3; ++a) {
+      if (!o[a]) continue;
+      int cls = g->desc.face_bc[2 * a + (o[a] > 0 ? 1 : 0)];
+      int pr = bc_priority(g->bc_host[cls].kind);
+      if (pr > bp) { bp = pr; best = cls; }
+    }
+    g->face_host[i] = (uint8_t)best;
+  }
+}
+
+size_t pop_bytes(const lbm_grid* g, int L) { return (size_t)g->host[L].nfluid * g->Q * kCells * g->tsize; }
+
+LevelView view_of(const lbm_grid* g, int L) {
+  LevelView v{};
+  if (L < 0 || L >= g->levels) return v;
+  const HostLevel& H = g->host[L];
+  for (int a = 0; a < 3; ++a) { v.n[a] = (int32_t)H.n[a]; v.nb[a] = H.nb[a]; }
+  v.blkmap = g->dev[L].blkmap;
+  v.types = g->dev[L].types;
+  return v;
+}
+
+template <typename T>
+StepParams<T> make_params(const lbm_grid* g, int L, int64_t k) {
+  StepParams<T> p{};
+  const DevLevel& D = g->dev[L];
+  p.own = view_of(g, L);
+  p.coarse = view_of(g, L - 1);
+  p.fine = view_of(g, L + 1);
+  p.nbr = D.nbr;
+  p.special_slot = D.special_slot;
+  p.cellinfo = D.cellinfo;
+  p.origin = D.origin;
+  p.src = static_cast<const T*>(D.pop[k & 1]);
+  p.dst = static_cast<T*>(D.pop[(k + 1) & 1]);
+  if (L > 0) p.csrc = static_cast<const T*>(g->dev[L - 1].pop[((k + 1) / 2) & 1]);
+  if (L + 1 < g->levels) {
+    p.fa = static_cast<const T*>(g->dev[L + 1].pop[1]);  // C_{L+1}^{2k-1}
+    p.fb = static_cast<const T*>(g->dev[L + 1].pop[0]);  // C_{L+1}^{2k}
+  }
+  p.bc = g->bc_dev;
+  p.omega = (T)g->omega[L];
+  for (int a = 0; a < 3; ++a) p.periodic[a] = g->desc.periodic[a];
+  p.face_cls = g->face_dev;
+  p.nfluid = g->host[L].nfluid;
+  return p;
+}
+
+void launch_F(lbm_grid* g, int L, int64_t k, int kind) {
+  if (g->prec == LBM_FP32) {
+    StepParams<float> p = make_params<float>(g, L, k);
+    launch_level_step(g->Q, g->coll, g->prec, kind, &p, g->stream);
+  } else {
+    StepParams<double> p = make_params<double>(g, L, k);
+    launch_level_step(g->Q, g->coll, g->prec, kind, &p, g->stream);
+  }
+}
+
+// The pipelined order of one coarse step n (0-based): list of (L, k).
+void step_order(int levels, int64_t n, std::vector<std::pair<int, int64_t>>& out) {
+  out.clear();
+  const int F = levels - 1;
+  const int64_t per = (int64_t)1 << F;
+  for (int64_t k = per * n + 1; k <= per * (n + 1); ++k) {
+    out.push_back({F, k});
+    int L = F;
+    int64_t kk = k;
+    while (L > 0 && (kk & 1)) {
+      kk = (kk + 1) / 2;
+      --L;
+      out.push_back({L, kk});
+    }
+  }
+}
+
+lbm_status run_prologue(lbm_grid* g) {
+  // C_L^1 = Collision of the initial post-streaming state (buf 0 -> buf 1)
+  for (int L = 0; L < g->levels; ++L) launch_F(g, L, 0, 1);
+  CUDA_TRY(cudaGetLastError());
+  g->needs_prologue = false;
+  return LBM_OK;
+}
+
+lbm_status build_graphs(lbm_grid* g) {
+  std::vector<std::pair<int, int64_t>> order;
+  for (int par = 0; par < 2; ++par) {
+    if (g->graph[par]) continue;
+    step_order(g->levels, par, order);
+    cudaGraph_t graph;
+    CUDA_TRY(cudaStreamBeginCapture(g->stream, cudaStreamCaptureModeThreadLocal));
+    for (auto& lk : order) launch_F(g, lk.first, lk.second, 0);
+    cudaError_t le = cudaGetLastError();
+    CUDA_TRY(cudaStreamEndCapture(g->stream, &graph));
+    if (le != cudaSuccess) return fail(LBM_E_CUDA, std::string("capture: ") + cudaGetErrorString(le));
+    cudaError_t e = cudaGraphInstantiate(&g->graph[par], graph, 0);
+    cudaGraphDestroy(graph);
+    if (e != cudaSuccess) return fail(LBM_E_CUDA, std::string("cudaGraphInstantiate: ") + cudaGetErrorString(e));
+  }
+  return LBM_OK;
+}
+
+int cur_buf(const lbm_grid* g, int L) {
+  if (g->needs_prologue) return 0;
+  // C_L^{k+1} with k = 2^L * steps
+  const int64_t k = (g->steps << L);
+  return (int)((k + 1) & 1);
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* lbm_last_error(void) { return g_err.c_str(); }
+
+const char* lbm_version(void) { return "lbmr 0.1 (sm_100a)"; }
+
+lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t* const* masks, lbm_grid** out) {
+  g_err.clear();
+  if (!d || !masks || !out) return fail(LBM_E_INVAL, "NULL argument");
+  *out = nullptr;
+  if (levels < 1 || levels > 16) return fail(LBM_E_INVAL, "levels must be in [1,16]");
+  if (d->nx < 1 || d->ny < 1 || d->nz < 1) return fail(LBM_E_INVAL, "nx, ny, nz must be >= 1");
+  for (int L = 0; L < levels; ++L)
+    if (!masks[L]) return fail(LBM_E_INVAL, "masks[" + std::to_string(L) + "] is NULL");
+  if (d->lattice != LBM_D3Q19 && d->lattice != LBM_D3Q27) return fail(LBM_E_INVAL, "lattice must be 19 or 27");
+  if (d->collision != LBM_BGK && d->collision != LBM_KBC) return fail(LBM_E_INVAL, "bad collision");
+  if (d->precision != LBM_FP32 && d->precision != LBM_FP64) return fail(LBM_E_INVAL, "bad precision");
+  if (d->collision == LBM_KBC && d->lattice != LBM_D3Q27)
+    return fail(LBM_E_UNSUPPORTED, "KBC requires D3Q27 (P:L260)");
+  if (!(d->omega0 > 0.0 && d->omega0 < 2.0)) return fail(LBM_E_INVAL, "omega0 must be in (0, 2)");
+  for (int a = 0; a < 3; ++a) {
+    if (d->periodic[a]) continue;
+    for (int s = 0; s < 2; ++s) {
+      int c = d->face_bc[2 * a + s];
+      if (c < 2 || c > 254) return fail(LBM_E_INVAL, "face_bc of a non-periodic face must be a BC class in 2..254");
+    }
+  }
+  if (d->n_ranks > 1) return fail(LBM_E_UNSUPPORTED, "multi-rank slab partition not enabled in this build");
+  for (int L = 0; L < levels; ++L) {
+    int64_t n0 = (int64_t)d->nx << L, n1 = (int64_t)d->ny << L, n2 = (int64_t)d->nz << L;
+    if (n0 > (1 << 28) || n1 > (1 << 28) || n2 > (1 << 28)) return fail(LBM_E_INVAL, "level too large");
+  }
+
+  lbm_grid* g = new lbm_grid();
+  g->desc = *d;
+  g->levels = levels;
+  g->Q = d->lattice;
+  g->coll = d->collision;
+  g->prec = d->precision;
+  g->tsize = d->precision == LBM_FP32 ? 4 : 8;
+  for (int c = 0; c < 256; ++c) {
+    g->bc_host[c].kind = LBM_BC_NOSLIP;
+    g->bc_host[c].pad_ = 0;
+    g->bc_host[c].u[0] = g->bc_host[c].u[1] = g->bc_host[c].u[2] = 0.0;
+  }
+  BuildInput in{};
+  in.n0[0] = d->nx; in.n0[1] = d->ny; in.n0[2] = d->nz;
+  for (int a = 0; a < 3; ++a) in.periodic[a] = d->periodic[a] ? 1 : 0;
+  in.levels = levels;
+  in.Q = g->Q;
+  in.masks = masks;
+  std::string err;
+  int st = build_grid(in, g->host, err);
+  if (st) {
+    delete g;
+    return fail((lbm_status)st, err);
+  }
+  for (int L = 0; L < levels; ++L) g->omega.push_back(omega_level(d->omega0, L));
+
+  auto cleanup = [&](lbm_status s) {
+    std::string keep = g_err;
+    lbm_grid_destroy(g);
+    g_err = keep;
+    return s;
+  };
+  if (d->stream) {
+    g->stream = static_cast<cudaStream_t>(d->stream);
+  } else {
+    if (cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking) != cudaSuccess) {
+      delete g;
+      return fail(LBM_E_CUDA, "cudaStreamCreate failed (no CUDA device?)");
+    }
+    g->own_stream = true;
+  }
+  g->dev.resize(levels);
+  lbm_status s;
+  for (int L = 0; L < levels; ++L) {
+    HostLevel& H = g->host[L];
+    DevLevel& D = g->dev[L];
+    if ((s = dev_upload(g, &D.blkmap, H.blkmap))) return cleanup(s);
+    if ((s = dev_upload(g, &D.types, H.types))) return cleanup(s);
+    if ((s = dev_upload(g, &D.origin, H.origin))) return cleanup(s);
+    if ((s = dev_upload(g, &D.nbr, H.nbr))) return cleanup(s);
+    if ((s = dev_upload(g, &D.special_slot, H.special_slot))) return cleanup(s);
+    if ((s = dev_upload(g, &D.cellinfo, H.cellinfo))) return cleanup(s);
+    for (int b = 0; b < 2; ++b) {
+      if ((s = dev_alloc(g, &D.pop[b], pop_bytes(g, L)))) return cleanup(s);
+      if (cudaMemset(D.pop[b], 0, pop_bytes(g, L)) != cudaSuccess) return cleanup(fail(LBM_E_CUDA, "memset"));
+    }
+    // the dense per-level tables are on the device now; keep only counters
+    std::vector<int32_t>().swap(H.blkmap);
+    std::vector<uint32_t>().swap(H.cellinfo);
+    std::vector<int32_t>().swap(H.nbr);
+  }
+  void* p;
+  if ((s = dev_alloc(g, &p, sizeof(BCEntry) * 256))) return cleanup(s);
+  g->bc_dev = static_cast<BCEntry*>(p);
+  if ((s = dev_alloc(g, &p, 32))) return cleanup(s);
+  g->face_dev = static_cast<uint8_t*>(p);
+  compute_face_classes(g);
+  if (cudaMemcpy(g->bc_dev, g->bc_host, sizeof(g->bc_host), cudaMemcpyHostToDevice) != cudaSuccess ||
+      cudaMemcpy(g->face_dev, g->face_host, 27, cudaMemcpyHostToDevice) != cudaSuccess)
+    return cleanup(fail(LBM_E_CUDA, "upload BC table"));
+  // populations start as g = 0, i.e. f = w (rest equilibrium, rho = 1)
+  g->needs_prologue = true;
+  *out = g;
+  return LBM_OK;
+}
+
+lbm_status lbm_set_bc(lbm_grid* g, int32_t cls, int32_t kind, const double* u) {
+  g_err.clear();
+  if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  if (cls < 2 || cls > 254) return fail(LBM_E_INVAL, "bc_class must be in 2..254");
+  if (kind != LBM_BC_NOSLIP && kind != LBM_BC_VELOCITY && kind != LBM_BC_OUTFLOW)
+    return fail(LBM_E_INVAL, "bad BC kind");
+  g->bc_host[cls].kind = kind;
+  for (int a = 0; a < 3; ++a) g->bc_host[cls].u[a] = u ? u[a] : 0.0;
+  compute_face_classes(g);
+  CUDA_TRY(cudaMemcpyAsync(g->bc_dev + cls, g->bc_host + cls, sizeof(BCEntry), cudaMemcpyHostToDevice, g->stream));
+  CUDA_TRY(cudaMemcpyAsync(g->face_dev, g->face_host, 27, cudaMemcpyHostToDevice, g->stream));
+  return LBM_OK;
+}
+
+static lbm_status init_level(lbm_grid* g, int L, const double* rho, const double* u, double rho0, const double* u0) {
+  const HostLevel& H = g->host[L];
+  const size_t ncell = (size_t)H.nfluid * kCells;
+  std::vector<double> r(ncell, rho0), v(ncell * 3, 0.0);
+  if (u0)
+    for (size_t c = 0; c < ncell; ++c) { v[3 * c] = u0[0]; v[3 * c + 1] = u0[1]; v[3 * c + 2] = u0[2]; }
+  if (rho || u) {
+#pragma omp parallel for schedule(static)
+    for (int32_t b = 0; b < H.nfluid; ++b) {
+      const int64_t ox = (int64_t)H.origin[3 * b] * kBlock, oy = (int64_t)H.origin[3 * b + 1] * kBlock,
+                    oz = (int64_t)H.origin[3 * b + 2] * kBlock;
+      for (int l = 0; l < kCells; ++l) {
+        if (H.types[(size_t)b * kCells + l] != kFluid) continue;
+        const int64_t x = ox + (l & 7), y = oy + ((l >> 3) & 7), z = oz + (l >> 6);
+        const int64_t c = (x * H.n[1] + y) * H.n[2] + z;
+        const size_t k = (size_t)b * kCells + l;
+        if (rho) r[k] = rho[c];
+        if (u) { v[3 * k] = u[3 * c]; v[3 * k + 1] = u[3 * c + 1]; v[3 * k + 2] = u[3 * c + 2]; }
+      }
+    }
+  }
+  double *dr = nullptr, *du = nullptr;
+  CUDA_TRY(cudaMalloc(&dr, std::max<size_t>(ncell, 1) * sizeof(double)));
+  CUDA_TRY(cudaMalloc(&du, std::max<size_t>(ncell, 1) * 3 * sizeof(double)));
+  CUDA_TRY(cudaMemcpyAsync(dr, r.data(), ncell * sizeof(double), cudaMemcpyHostToDevice, g->stream));
+  CUDA_TRY(cudaMemcpyAsync(du, v.data(), ncell * 3 * sizeof(double), cudaMemcpyHostToDevice, g->stream));
+  launch_init_eq(g->Q, g->prec, g->dev[L].pop[0], g->dev[L].types, H.nfluid, dr, du, g->stream);
+  CUDA_TRY(cudaGetLastError());
+  CUDA_TRY(cudaStreamSynchronize(g->stream));
+  cudaFree(dr);
+  cudaFree(du);
+  return LBM_OK;
+}
+
+lbm_status lbm_init_equilibrium(lbm_grid* g, int32_t level, const double* rho, const double* u) {
+  g_err.clear();
+  if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  if (g->broken) return fail(LBM_E_STATE, "grid is in an error state");
+  if (level < 0 || level >= g->levels) return fail(LBM_E_INVAL, "level out of range");
+  if (g->init_locked)
+    return fail(LBM_E_STATE, "lbm_init_equilibrium after lbm_step: call lbm_init_uniform first");
+  lbm_status s = init_level(g, level, rho, u, 1.0, nullptr);
+  if (s) return s;
+  g->needs_prologue = true;
+  g->steps = 0;
+  return LBM_OK;
+}
+
+lbm_status lbm_init_uniform(lbm_grid* g, double rho0, const double* u0) {
+  g_err.clear();
+  if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  if (g->broken) return fail(LBM_E_STATE, "grid is in an error state");
+  for (int L = 0; L < g->levels; ++L) {
+    lbm_status s = init_level(g, L, nullptr, nullptr, rho0, u0);
+    if (s) return s;
+  }
+  g->needs_prologue = true;
+  g->init_locked = false;
+  g->steps = 0;
+  return LBM_OK;
+}
+
+lbm_status lbm_step(lbm_grid* g, int32_t n) {
+  g_err.clear();
+  if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  if (g->broken) return fail(LBM_E_STATE, "grid is in an error state");
+  if (n < 0) return fail(LBM_E_INVAL, "n_coarse must be >= 0");
+  if (n == 0) return LBM_OK;
+  lbm_status s;
+  if (g->needs_prologue && (s = run_prologue(g))) { g->broken = true; return s; }
+  if ((s = build_graphs(g))) { g->broken = true; return s; }
+  for (int i = 0; i < n; ++i) {
+    cudaError_t e = cudaGraphLaunch(g->graph[g->steps & 1], g->stream);
+    if (e != cudaSuccess) {
+      g->broken = true;
+      return fail(LBM_E_CUDA, std::string("cudaGraphLaunch: ") + cudaGetErrorString(e));
+    }
+    ++g->steps;
+  }
+  g->init_locked = true;
+  return LBM_OK;
+}
+
+lbm_status lbm_profile_levels(lbm_grid* g, int32_t n, double* ms_per_level, int64_t* launches_per_level) {
+  g_err.clear();
+  if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  if (g->broken) return fail(LBM_E_STATE, "grid is in an error state");
+  lbm_status s;
+  if (g->needs_prologue && (s = run_prologue(g))) return s;
+  std::vector<std::pair<int, int64_t>> order;
+  std::vector<cudaEvent_t> ev;
+  std::vector<int> lev;
+  for (int i = 0; i < n; ++i) {
+    step_order(g->levels, g->steps, order);
+    for (auto& lk : order) {
+      cudaEvent_t a, b;
+      CUDA_TRY(cudaEventCreate(&a));
+      CUDA_TRY(cudaEventCreate(&b));
+      CUDA_TRY(cudaEventRecord(a, g->stream));
+      launch_F(g, lk.first, lk.second, 0);
+      CUDA_TRY(cudaEventRecord(b, g->stream));
+      ev.push_back(a);
+      ev.push_back(b);
+      lev.push_back(lk.first);
+    }
+    ++g->steps;
+  }
+  CUDA_TRY(cudaGetLastError());
+  CUDA_TRY(cudaStreamSynchronize(g->stream));
+  std::vector<double> ms(g->levels, 0.0);
+  std::vector<int64_t> cnt(g->levels, 0);
+  for (size_t i = 0; i < lev.size(); ++i) {
+    float t = 0;
+    CUDA_TRY(cudaEventElapsedTime(&t, ev[2 * i], ev[2 * i + 1]));
+    ms[lev[i]] += t;
+    cnt[lev[i]] += 1;
+  }
+  for (auto e : ev) cudaEventDestroy(e);
+  for (int L = 0; L < g->levels; ++L) {
+    if (ms_per_level) ms_per_level[L] = ms[L];
+    if (launches_per_level) launches_per_level[L] = cnt[L];
+  }
+  g->init_locked = true;
+  return LBM_OK;
+}
+
+lbm_status lbm_synchronize(lbm_grid* g) {
+  g_err.clear();
+  if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  CUDA_TRY(cudaStreamSynchronize(g->stream));
+  return LBM_OK;
+}
+
+lbm_status lbm_macroscopic(lbm_grid* g, int32_t L, double* rho, double* u) {
+  g_err.clear();
+  if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  if (L < 0 || L >= g->levels) return fail(LBM_E_INVAL, "level out of range");
+  const HostLevel& H = g->host[L];
+  const size_t ncell = (size_t)H.nfluid * kCells;
+  double *dr = nullptr, *du = nullptr;
+  CUDA_TRY(cudaStreamSynchronize(g->stream));
+  CUDA_TRY(cudaMalloc(&dr, std::max<size_t>(ncell, 1) * sizeof(double)));
+  CUDA_TRY(cudaMalloc(&du, std::max<size_t>(ncell, 1) * 3 * sizeof(double)));
+  launch_macroscopic(g->Q, g->prec, g->dev[L].pop[cur_buf(g, L)], g->dev[L].types, H.nfluid, dr, du, nullptr,
+                     g->stream);
+  std::vector<double> r(ncell), v(3 * ncell);
+  CUDA_TRY(cudaGetLastError());
+  CUDA_TRY(cudaMemcpyAsync(r.data(), dr, ncell * sizeof(double), cudaMemcpyDeviceToHost, g->stream));
+  CUDA_TRY(cudaMemcpyAsync(v.data(), du, 3 * ncell * sizeof(double), cudaMemcpyDeviceToHost, g->stream));
+  CUDA_TRY(cudaStreamSynchronize(g->stream));
+  cudaFree(dr);
+  cudaFree(du);
+  const int64_t N = H.n[0] * H.n[1] * H.n[2];
+  const double nan = std::nan("");
+  if (rho) std::fill(rho, rho + N, nan);
+  if (u) std::fill(u, u + 3 * N, nan);
+#pragma omp parallel for schedule(static)
+  for (int32_t b = 0; b < H.nfluid; ++b) {
+    const int64_t ox = (int64_t)H.origin[3 * b] * kBlock, oy = (int64_t)H.origin[3 * b + 1] * kBlock,
+                  oz = (int64_t)H.origin[3 * b + 2] * kBlock;
+    for (int l = 0; l < kCells; ++l) {
+      if (H.types[(size_t)b * kCells + l] != kFluid) continue;
+      const int64_t x = ox + (l & 7), y = oy + ((l >> 3) & 7), z = oz + (l >> 6);
+      const int64_t c = (x * H.n[1] + y) * H.n[2] + z;
+      const size_t k = (size_t)b * kCells + l;
+      if (rho) rho[c] = r[k];
+      if (u) { u[3 * c] = v[3 * k]; u[3 * c + 1] = v[3 * k + 1]; u[3 * c + 2] = v[3 * k + 2]; }
+    }
+  }
+  return LBM_OK;
+}
+
+lbm_status lbm_stats(lbm_grid* g, int64_t* leaves, double* mass) {
+  g_err.clear();
+  if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  if (leaves)
+    for (int L = 0; L < g->levels; ++L) leaves[L] = g->host[L].leaves;
+  if (!mass) return LBM_OK;
+  double total = 0.0;
+  for (int L = 0; L < g->levels; ++L) {
+    const HostLevel& H = g->host[L];
+    double* bm = nullptr;
+    CUDA_TRY(cudaMalloc(&bm, std::max<int32_t>(H.nfluid, 1) * sizeof(double)));
+    launch_macroscopic(g->Q, g->prec, g->dev[L].pop[cur_buf(g, L)], g->dev[L].types, H.nfluid, nullptr, nullptr,
+                       bm, g->stream);
+    std::vector<double> h(H.nfluid);
+    CUDA_TRY(cudaGetLastError());
+    CUDA_TRY(cudaMemcpyAsync(h.data(), bm, H.nfluid * sizeof(double), cudaMemcpyDeviceToHost, g->stream));
+    CUDA_TRY(cudaStreamSynchronize(g->stream));
+    cudaFree(bm);
+    double sL = 0.0;
+    for (double x : h) sL += x;
+    total += sL * std::ldexp(1.0, -3 * L);
+  }
+  *mass = total;
+  return LBM_OK;
+}
+
+lbm_status lbm_grid_get_info(const lbm_grid* g, lbm_grid_info* info) {
+  g_err.clear();
+  if (!g || !info) return fail(LBM_E_INVAL, "NULL argument");
+  std::memset(info, 0, sizeof(*info));
+  info->levels = g->levels;
+  info->Q = g->Q;
+  info->precision = g->prec;
+  info->kernels_per_step = (1 << g->levels) - 1;
+  for (int L = 0; L < g->levels; ++L) {
+    info->leaves[L] = g->host[L].leaves;
+    info->blocks[L] = g->host[L].nfluid;
+    info->special_blocks[L] = g->host[L].nspecial;
+    info->special_cells[L] = g->host[L].special_cells;
+    info->total_blocks[L] = g->host[L].nblocks;
+  }
+  info->device_bytes = g->device_bytes;
+  info->steps_done = g->steps;
+  return LBM_OK;
+}
+
+void lbm_grid_destroy(lbm_grid* g) {
+  if (!g) return;
+  if (g->stream) cudaStreamSynchronize(g->stream);
+  for (int p = 0; p < 2; ++p)
+    if (g->graph[p]) cudaGraphExecDestroy(g->graph[p]);
+  for (void* p : g->allocs) cudaFree(p);
+  if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
+  delete g;
+}
+
+}  // extern "C"

@@ -1,0 +1,59 @@
+// kernels.h — launch interface of the sm_100a kernels (level_step.cu) used by
+// the host runtime (capi.cpp).  No torch types; plain device pointers.
+#pragma once
+#include <cstdint>
+
+#include <cuda_runtime.h>
+
+namespace lbmr {
+
+// Geometry of one level as the kernels see it (all pointers are device).
+struct LevelView {
+  int32_t n[3];             // cells per axis
+  int32_t nb[3];            // blocks per axis
+  const int32_t* blkmap;    // dense block map, -1 = no block
+  const uint8_t* types;     // [nblocks][512] cell types (lattice.h codes)
+};
+
+struct BCEntry {
+  int32_t kind;             // LBM_BC_NOSLIP / VELOCITY / OUTFLOW
+  int32_t pad_;
+  double u[3];              // wall / inlet velocity
+};
+
+// Parameters of one fused level-substep launch F_L^k: stream substep k of
+// level L (pull, with BC, Explosion from L-1 and Coalescence from L+1), then
+// collide substep k+1.
+template <typename T>
+struct StepParams {
+  LevelView own, coarse, fine;
+  const int32_t* nbr;           // [nfluid][27]
+  const int32_t* special_slot;  // [nfluid]
+  const uint32_t* cellinfo;     // [nspecial][512]
+  const int32_t* origin;        // [nblocks][3] block coordinates
+  const T* src;                 // C_L^k            [nfluid][Q][512]
+  T* dst;                       // C_L^{k+1}
+  const T* csrc;                // C_{L-1}^{ceil(k/2)}   (nullptr at L = 0)
+  const T* fa;                  // C_{L+1}^{2k-1}        (nullptr at the finest level)
+  const T* fb;                  // C_{L+1}^{2k}
+  const BCEntry* bc;            // [256]
+  T omega;                      // ω_L (Eq.9)
+  int32_t periodic[3];
+  const uint8_t* face_cls;      // [27] BC class of an out-of-domain source, by outside pattern
+  int32_t nfluid;
+};
+
+// kind: 0 = fused stream+collide, 1 = collide only (prologue C_L^1)
+void launch_level_step(int Q, int collision, int precision, int kind, const void* params, cudaStream_t s);
+
+// g = f^eq(rho,u) - w on the fluid cells of `nfluid` blocks; rho/u compact
+// device arrays [nfluid*512] and [nfluid*512*3] (double).
+void launch_init_eq(int Q, int precision, void* pop, const uint8_t* types, int32_t nfluid,
+                    const double* rho, const double* u, cudaStream_t s);
+
+// rho/u (double, compact, NaN on non-fluid cells) of the post-collision
+// buffer `pop`; optional per-block mass partial sums block_mass[nfluid].
+void launch_macroscopic(int Q, int precision, const void* pop, const uint8_t* types, int32_t nfluid,
+                        double* rho, double* u, double* block_mass, cudaStream_t s);
+
+}  // namespace lbmr

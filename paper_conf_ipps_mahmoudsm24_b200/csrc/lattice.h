@@ -1,0 +1,50 @@
+// lattice.h — D3Q19 / D3Q27 velocity sets of the product path (host + device).
+// P:L37 §II names the lattices; weights are the standard ones (Krüger et al.,
+// ref [2] of the paper).  Ordering: rest, then opposite pairs (q, q+1) with
+// q odd, so opp(q) = q + 1 for odd q and q - 1 for even q > 0.  D3Q19 is the
+// 19-entry prefix of D3Q27.
+#pragma once
+
+#ifdef __CUDACC__
+#define LBM_HD __host__ __device__
+#else
+#define LBM_HD
+#endif
+
+namespace lbmr {
+
+// e_x, e_y, e_z of each direction (the lists are reused for __constant__ copies)
+#define LBMR_EX_LIST 0, 1, -1, 0, 0, 0, 0, 1, -1, 1, -1, 1, -1, 1, -1, 0, 0, 0, 0, 1, -1, 1, -1, 1, -1, -1, 1
+#define LBMR_EY_LIST 0, 0, 0, 1, -1, 0, 0, 1, -1, -1, 1, 0, 0, 0, 0, 1, -1, 1, -1, 1, -1, 1, -1, -1, 1, 1, -1
+#define LBMR_EZ_LIST 0, 0, 0, 0, 0, 1, -1, 0, 0, 0, 0, 1, -1, -1, 1, 1, -1, -1, 1, 1, -1, -1, 1, 1, -1, 1, -1
+constexpr int kEx[27] = {LBMR_EX_LIST};
+constexpr int kEy[27] = {LBMR_EY_LIST};
+constexpr int kEz[27] = {LBMR_EZ_LIST};
+
+// compile-time accessors (fold to constants inside unrolled loops)
+LBM_HD constexpr int ex(int q) { constexpr int t[27] = {LBMR_EX_LIST}; return t[q]; }
+LBM_HD constexpr int ey(int q) { constexpr int t[27] = {LBMR_EY_LIST}; return t[q]; }
+LBM_HD constexpr int ez(int q) { constexpr int t[27] = {LBMR_EZ_LIST}; return t[q]; }
+
+LBM_HD constexpr int opp(int q) { return q == 0 ? 0 : ((q & 1) ? q + 1 : q - 1); }
+
+template <int Q>
+LBM_HD constexpr double weight(int q) {
+  return Q == 19 ? (q == 0 ? 1.0 / 3.0 : q < 7 ? 1.0 / 18.0 : 1.0 / 36.0)
+                 : (q == 0 ? 8.0 / 27.0 : q < 7 ? 2.0 / 27.0 : q < 19 ? 1.0 / 54.0 : 1.0 / 216.0);
+}
+
+// neighbour-block slot of an offset (dx,dy,dz) in {-1,0,1}^3
+LBM_HD constexpr int nbr_slot(int dx, int dy, int dz) { return (dx + 1) + 3 * (dy + 1) + 9 * (dz + 1); }
+
+constexpr int kBlock = 8;            // B = 8 (B compile time)
+constexpr int kCells = 512;          // B^3
+constexpr unsigned kFluidBit = 1u << 31;
+
+// cell type codes stored per block (mask codes + derived states)
+constexpr unsigned char kAbsent = 0;    // covered by a coarser leaf, or outside the domain
+constexpr unsigned char kFluid = 1;
+constexpr unsigned char kRefined = 255; // covered by finer leaves
+// 2..254: boundary-condition leaf of that class
+
+}  // namespace lbmr

@@ -1,0 +1,401 @@
+// level_step.cu — sm_100a kernels of the multi-level LBM hot path.
+//
+// F_L^k (level_step_kernel): ONE fused kernel per level-substep.  For every
+// fluid leaf p of level L it pulls the Q populations of substep k
+//   * Streaming, Eq.(2): same-level source p - e_q, via the 8^3 block's
+//     neighbour table;
+//   * Explosion, Eq.(10): source inside a coarser leaf -> that leaf's
+//     post-collision value C_{L-1}^{ceil(k/2)} (reading R-A1; both fine
+//     substeps read the same coarse value, R-A4; the fine level reads the
+//     coarse grid directly);
+//   * Coalescence, Eq.(11), gather form of Accumulate: source
+//     cell refined -> (sum_B C_{L+1}^{2k-1} + sum_B C_{L+1}^{2k}) / (2|B|) over
+//     the fine fluid leaves beta with beta + e_q inside p (R-A2, R-A3);
+//   * bounce-back / moving wall / outflow (R-A11);
+// then collides (BGK Eq.(3)/(5), or KBC [18] per R-A9) with ω_L (Eq.9) and
+// writes C_L^{k+1}.  Populations are stored shifted, g = f - w (R-A16), in
+// AoSoA layout [block][q][512] so every same-level pull of a warp is
+// a 128-byte-coalesced row load.
+//
+// The CTA is half an 8^3 block (256 threads, one cell each).  Links whose
+// source is not a same-level fluid leaf reachable by the block arithmetic are
+// flagged per cell by the host builder (cellinfo) and resolved in
+// slow_link(); blocks without such cells (the bulk) never read cellinfo.
+#include <cmath>
+#include <cstdio>
+
+#include "../../include/lbmr.h"
+#include "kernels.h"
+#include "lattice.h"
+
+namespace lbmr {
+
+__constant__ int c_ex[27] = {LBMR_EX_LIST};
+__constant__ int c_ey[27] = {LBMR_EY_LIST};
+__constant__ int c_ez[27] = {LBMR_EZ_LIST};
+
+template <int Q>
+__device__ __forceinline__ double wq_rt(int q) {
+  // runtime-q weight (slow path only)
+  if (Q == 19) return q == 0 ? 1.0 / 3.0 : (q < 7 ? 1.0 / 18.0 : 1.0 / 36.0);
+  return q == 0 ? 8.0 / 27.0 : (q < 7 ? 2.0 / 27.0 : (q < 19 ? 1.0 / 54.0 : 1.0 / 216.0));
+}
+
+template <typename T>
+__device__ __forceinline__ T nan_of() {
+  return T(NAN);
+}
+
+// ---------------------------------------------------------------- collision
+// Moments of shifted populations: rho = 1 + sum g (Eq.6), j = sum e g (Eq.7).
+template <int Q, typename T>
+__device__ __forceinline__ void moments(const T (&g)[Q], T& drho, T& jx, T& jy, T& jz) {
+  drho = T(0); jx = T(0); jy = T(0); jz = T(0);
+#pragma unroll
+  for (int q = 0; q < Q; ++q) {
+    drho += g[q];
+    if (ex(q) > 0) jx += g[q]; else if (ex(q) < 0) jx -= g[q];
+    if (ey(q) > 0) jy += g[q]; else if (ey(q) < 0) jy -= g[q];
+    if (ez(q) > 0) jz += g[q]; else if (ez(q) < 0) jz -= g[q];
+  }
+}
+
+// shifted equilibrium g^eq_q = w_q (drho + rho (3 e.u + 4.5 (e.u)^2 - 1.5 u^2))
+template <int Q, typename T>
+__device__ __forceinline__ T geq(int q, T drho, T rho, T ux, T uy, T uz, T usq15) {
+  const T eu = T(ex(q)) * ux + T(ey(q)) * uy + T(ez(q)) * uz;
+  return T(weight<Q>(q)) * (drho + rho * (T(3) * eu + T(4.5) * eu * eu - usq15));
+}
+
+template <int Q, typename T>
+__device__ __forceinline__ void collide_bgk(T (&g)[Q], T omega) {
+  T drho, jx, jy, jz;
+  moments<Q, T>(g, drho, jx, jy, jz);
+  const T rho = T(1) + drho;
+  const T inv = T(1) / rho;
+  const T ux = jx * inv, uy = jy * inv, uz = jz * inv;
+  const T usq15 = T(1.5) * (ux * ux + uy * uy + uz * uz);
+#pragma unroll
+  for (int q = 0; q < Q; ++q) {
+    const T e = geq<Q, T>(q, drho, rho, ux, uy, uz, usq15);
+    g[q] = g[q] - omega * (g[q] - e);
+  }
+}
+
+// KBC (reading R-A9) on shifted populations; D3Q27 only.
+template <typename T>
+__device__ __forceinline__ void collide_kbc(T (&g)[27], T omega) {
+  constexpr int Q = 27;
+  T drho, jx, jy, jz;
+  moments<Q, T>(g, drho, jx, jy, jz);
+  const T rho = T(1) + drho;
+  const T inv = T(1) / rho;
+  const T ux = jx * inv, uy = jy * inv, uz = jz * inv;
+  const T usq15 = T(1.5) * (ux * ux + uy * uy + uz * uz);
+  // g <- f^neq = g - g^eq ; second moments of f^neq
+  T pxx = 0, pyy = 0, pzz = 0, pxy = 0, pxz = 0, pyz = 0;
+#pragma unroll
+  for (int q = 0; q < Q; ++q) {
+    g[q] -= geq<Q, T>(q, drho, rho, ux, uy, uz, usq15);
+    if (ex(q)) pxx += g[q];
+    if (ey(q)) pyy += g[q];
+    if (ez(q)) pzz += g[q];
+    if (ex(q) * ey(q) > 0) pxy += g[q]; else if (ex(q) * ey(q) < 0) pxy -= g[q];
+    if (ex(q) * ez(q) > 0) pxz += g[q]; else if (ex(q) * ez(q) < 0) pxz -= g[q];
+    if (ey(q) * ez(q) > 0) pyz += g[q]; else if (ey(q) * ez(q) < 0) pyz -= g[q];
+  }
+  const T nxz = pxx - pzz, nyz = pyy - pzz;
+  const T sx = (T(2) * nxz - nyz) / T(6), sy = (-nxz + T(2) * nyz) / T(6), sz = (-nxz - nyz) / T(6);
+  const T exy = pxy / T(4), exz = pxz / T(4), eyz = pyz / T(4);
+  auto ds = [&](int q) -> T {
+    const int n2 = ex(q) * ex(q) + ey(q) * ey(q) + ez(q) * ez(q);
+    if (n2 == 1) return ex(q) ? sx : (ey(q) ? sy : sz);
+    if (n2 == 2) {
+      if (ez(q) == 0) return T(ex(q) * ey(q)) * exy;
+      if (ey(q) == 0) return T(ex(q) * ez(q)) * exz;
+      return T(ey(q) * ez(q)) * eyz;
+    }
+    return T(0);
+  };
+  T sh = 0, hh = 0;
+#pragma unroll
+  for (int q = 0; q < Q; ++q) {
+    const T feq = T(weight<Q>(q)) + geq<Q, T>(q, drho, rho, ux, uy, uz, usq15);
+    const T s = ds(q);
+    const T h = g[q] - s;
+    sh += s * h / feq;
+    hh += h * h / feq;
+  }
+  const T beta = omega / T(2);
+  const T gamma = (hh < T(1e-30)) ? T(2) : T(1) / beta - (T(2) - T(1) / beta) * sh / hh;
+#pragma unroll
+  for (int q = 0; q < Q; ++q) {
+    const T s = ds(q);
+    const T h = g[q] - s;
+    const T e = geq<Q, T>(q, drho, rho, ux, uy, uz, usq15);
+    g[q] = (g[q] + e) - beta * (T(2) * s + gamma * h);
+  }
+}
+
+template <int Q, int COLL, typename T>
+__device__ __forceinline__ void collide(T (&g)[Q], T omega) {
+  if constexpr (COLL == LBM_KBC && Q == 27) collide_kbc<T>(g, omega);
+  else collide_bgk<Q, T>(g, omega);
+}
+
+// ---------------------------------------------------------------- slow links
+__device__ __forceinline__ int lookup(const LevelView& v, int x, int y, int z, int& local) {
+  local = (x & 7) | ((y & 7) << 3) | ((z & 7) << 6);
+  return __ldg(v.blkmap + ((size_t)(x >> 3) * v.nb[1] + (y >> 3)) * v.nb[2] + (z >> 3));
+}
+
+__device__ __forceinline__ unsigned type_at(const LevelView& v, int b, int local) {
+  return b < 0 ? kAbsent : __ldg(v.types + (size_t)b * kCells + local);
+}
+
+__device__ __forceinline__ bool is_bc(unsigned t) { return t != kAbsent && t != kFluid && t != kRefined; }
+
+// BC rule for pulled link q of the cell (blk, t): halfway bounce-back of the
+// cell's own post-collision opposite population, + 6 w_q rho_w e_q.u_w for a
+// moving wall / inlet, g = 0 (f = w_q) for outflow.
+template <int Q, typename T>
+__device__ __forceinline__ T bc_value(const StepParams<T>& P, unsigned cls, int q, int blk, int t) {
+  const int kind = __ldg(&P.bc[cls].kind);
+  if (kind == LBM_BC_OUTFLOW) return T(0);
+  const int o = (q == 0) ? 0 : ((q & 1) ? q + 1 : q - 1);
+  T v = __ldg(P.src + ((size_t)blk * Q + o) * kCells + t);
+  if (kind == LBM_BC_VELOCITY) {
+    const double eu = c_ex[q] * __ldg(&P.bc[cls].u[0]) + c_ey[q] * __ldg(&P.bc[cls].u[1]) +
+                      c_ez[q] * __ldg(&P.bc[cls].u[2]);
+    v += T(6.0 * wq_rt<Q>(q) * 1.0 * eu);
+  }
+  return v;
+}
+
+template <int Q, typename T>
+__device__ __forceinline__ T slow_link(const StepParams<T>& P, int q, int blk, int t, int px, int py, int pz) {
+  const int exq = c_ex[q], eyq = c_ey[q], ezq = c_ez[q];
+  int s[3] = {px - exq, py - eyq, pz - ezq};
+  int out[3] = {0, 0, 0};
+  bool outside = false;
+#pragma unroll
+  for (int a = 0; a < 3; ++a) {
+    const int n = P.own.n[a];
+    if (s[a] < 0 || s[a] >= n) {
+      if (P.periodic[a]) s[a] += (s[a] < 0) ? n : -n;
+      else { out[a] = (s[a] < 0) ? -1 : 1; outside = true; }
+    }
+  }
+  if (outside) return bc_value<Q, T>(P, __ldg(P.face_cls + (out[0] + 1) + 3 * (out[1] + 1) + 9 * (out[2] + 1)), q, blk, t);
+  int tl;
+  int b = lookup(P.own, s[0], s[1], s[2], tl);
+  unsigned ty = type_at(P.own, b, tl);
+  if (ty == kFluid) return __ldg(P.src + ((size_t)b * Q + q) * kCells + tl);  // Eq.(2)
+  if (is_bc(ty)) return bc_value<Q, T>(P, ty, q, blk, t);
+  if (ty == kAbsent) {
+    // Explosion, Eq.(10): the coarser leaf containing s
+    int cl;
+    const int cb = lookup(P.coarse, s[0] >> 1, s[1] >> 1, s[2] >> 1, cl);
+    const unsigned ct = type_at(P.coarse, cb, cl);
+    if (ct == kFluid) return __ldg(P.csrc + ((size_t)cb * Q + q) * kCells + cl);
+    if (is_bc(ct)) return bc_value<Q, T>(P, ct, q, blk, t);
+    return nan_of<T>();
+  }
+  // Coalescence, Eq.(11): fine fluid leaves beta = 2p - e_q + c, c in {0,1}^3
+  int64_t off[8];
+  int nB = 0;
+  unsigned firstbc = 0;
+#pragma unroll
+  for (int c = 0; c < 8; ++c) {
+    int f[3] = {2 * px - exq + (c >> 2), 2 * py - eyq + ((c >> 1) & 1), 2 * pz - ezq + (c & 1)};
+    bool ok = true;
+#pragma unroll
+    for (int a = 0; a < 3; ++a) {
+      const int n = P.fine.n[a];
+      if (f[a] < 0 || f[a] >= n) {
+        if (P.periodic[a]) f[a] += (f[a] < 0) ? n : -n;
+        else ok = false;
+      }
+    }
+    off[c] = -1;
+    if (!ok) continue;
+    int fl;
+    const int fbk = lookup(P.fine, f[0], f[1], f[2], fl);
+    const unsigned ft = type_at(P.fine, fbk, fl);
+    if (ft == kFluid) {
+      off[c] = ((int64_t)fbk * Q + q) * kCells + fl;
+      ++nB;
+    } else if (is_bc(ft) && firstbc == 0) {
+      firstbc = ft;
+    }
+  }
+  if (nB > 0) {
+    T acc = T(0);
+#pragma unroll
+    for (int c = 0; c < 8; ++c)
+      if (off[c] >= 0) acc += __ldg(P.fa + off[c]);
+#pragma unroll
+    for (int c = 0; c < 8; ++c)
+      if (off[c] >= 0) acc += __ldg(P.fb + off[c]);
+    return acc / T(2 * nB);
+  }
+  if (firstbc) return bc_value<Q, T>(P, firstbc, q, blk, t);
+  return nan_of<T>();
+}
+
+// ---------------------------------------------------------------- fused kernel
+template <int Q, int COLL, typename T, bool STREAM>
+__global__ void __launch_bounds__(256) level_step_kernel(const StepParams<T> P) {
+  __shared__ int s_nbr[27];
+  const int blk = blockIdx.x >> 1;
+  const int t = ((blockIdx.x & 1) << 8) | threadIdx.x;
+  if (STREAM && threadIdx.x < 27) s_nbr[threadIdx.x] = __ldg(P.nbr + (size_t)blk * 27 + threadIdx.x);
+  const int slot = __ldg(P.special_slot + blk);
+  uint32_t info = kFluidBit;
+  if (slot >= 0) info = __ldg(P.cellinfo + (size_t)slot * kCells + t);
+  if (STREAM) __syncthreads();
+  if (!(info & kFluidBit)) return;
+
+  const int lx = t & 7, ly = (t >> 3) & 7, lz = t >> 6;
+  T g[Q];
+  if (STREAM) {
+#pragma unroll
+    for (int q = 0; q < Q; ++q) {
+      const int sx = lx - ex(q), sy = ly - ey(q), sz = lz - ez(q);
+      const int nb = s_nbr[nbr_slot(sx >> 3, sy >> 3, sz >> 3)];
+      const int sl = (sx & 7) | ((sy & 7) << 3) | ((sz & 7) << 6);
+      g[q] = (info & (1u << q)) ? T(0) : __ldg(P.src + ((size_t)nb * Q + q) * kCells + sl);
+    }
+    uint32_t slow = info & ((1u << Q) - 1u);
+    if (slow) {
+      const int px = __ldg(P.origin + 3 * blk) * kBlock + lx;
+      const int py = __ldg(P.origin + 3 * blk + 1) * kBlock + ly;
+      const int pz = __ldg(P.origin + 3 * blk + 2) * kBlock + lz;
+      while (slow) {
+        const int q = __ffs(slow) - 1;
+        slow &= slow - 1;
+        const T v = slow_link<Q, T>(P, q, blk, t, px, py, pz);
+#pragma unroll
+        for (int qq = 0; qq < Q; ++qq)
+          if (qq == q) g[qq] = v;
+      }
+    }
+  } else {
+#pragma unroll
+    for (int q = 0; q < Q; ++q) g[q] = __ldg(P.src + ((size_t)blk * Q + q) * kCells + t);
+  }
+  collide<Q, COLL, T>(g, P.omega);
+  T* d = P.dst + (size_t)blk * Q * kCells + t;
+#pragma unroll
+  for (int q = 0; q < Q; ++q) d[(size_t)q * kCells] = g[q];
+}
+
+// ---------------------------------------------------------------- init / macroscopic
+template <int Q, typename T>
+__global__ void __launch_bounds__(512) init_eq_kernel(T* pop, const uint8_t* types, const double* rho,
+                                                      const double* u) {
+  const int blk = blockIdx.x, t = threadIdx.x;
+  const size_t c = (size_t)blk * kCells + t;
+  T* d = pop + (size_t)blk * Q * kCells + t;
+  if (types[c] != kFluid) {
+#pragma unroll
+    for (int q = 0; q < Q; ++q) d[(size_t)q * kCells] = T(0);
+    return;
+  }
+  const double r = rho[c], ux = u[3 * c], uy = u[3 * c + 1], uz = u[3 * c + 2];
+  const double usq15 = 1.5 * (ux * ux + uy * uy + uz * uz);
+#pragma unroll
+  for (int q = 0; q < Q; ++q) {
+    const double eu = ex(q) * ux + ey(q) * uy + ez(q) * uz;
+    // Eq.(5) minus w_q:  w_q (rho - 1 + rho (3 eu + 4.5 eu^2 - 1.5 u^2))
+    d[(size_t)q * kCells] = T(weight<Q>(q) * ((r - 1.0) + r * (3.0 * eu + 4.5 * eu * eu - usq15)));
+  }
+}
+
+template <int Q, typename T>
+__global__ void __launch_bounds__(512) macroscopic_kernel(const T* pop, const uint8_t* types, double* rho,
+                                                          double* u, double* block_mass) {
+  const int blk = blockIdx.x, t = threadIdx.x;
+  const size_t c = (size_t)blk * kCells + t;
+  double r = 0.0;
+  const bool fluid = types[c] == kFluid;
+  if (fluid) {
+    const T* s = pop + (size_t)blk * Q * kCells + t;
+    double d = 0, jx = 0, jy = 0, jz = 0;
+#pragma unroll
+    for (int q = 0; q < Q; ++q) {
+      const double g = (double)s[(size_t)q * kCells];
+      d += g;
+      jx += ex(q) * g;
+      jy += ey(q) * g;
+      jz += ez(q) * g;
+    }
+    r = 1.0 + d;
+    if (rho) rho[c] = r;
+    if (u) { u[3 * c] = jx / r; u[3 * c + 1] = jy / r; u[3 * c + 2] = jz / r; }
+  } else {
+    if (rho) rho[c] = NAN;
+    if (u) u[3 * c] = u[3 * c + 1] = u[3 * c + 2] = NAN;
+  }
+  if (block_mass) {
+    __shared__ double sm[16];
+    double v = r;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    if ((t & 31) == 0) sm[t >> 5] = v;
+    __syncthreads();
+    if (t == 0) {
+      double a = 0;
+      for (int i = 0; i < 16; ++i) a += sm[i];
+      block_mass[blk] = a;
+    }
+  }
+}
+
+// ---------------------------------------------------------------- dispatch
+template <int Q, int COLL, typename T>
+static void launch_typed(int kind, const void* params, cudaStream_t s) {
+  const StepParams<T>& p = *static_cast<const StepParams<T>*>(params);
+  if (p.nfluid <= 0) return;
+  dim3 grid(2 * p.nfluid), block(256);
+  if (kind == 0) level_step_kernel<Q, COLL, T, true><<<grid, block, 0, s>>>(p);
+  else level_step_kernel<Q, COLL, T, false><<<grid, block, 0, s>>>(p);
+}
+
+void launch_level_step(int Q, int collision, int precision, int kind, const void* params, cudaStream_t s) {
+  if (precision == LBM_FP32) {
+    if (Q == 19) launch_typed<19, LBM_BGK, float>(kind, params, s);
+    else if (collision == LBM_KBC) launch_typed<27, LBM_KBC, float>(kind, params, s);
+    else launch_typed<27, LBM_BGK, float>(kind, params, s);
+  } else {
+    if (Q == 19) launch_typed<19, LBM_BGK, double>(kind, params, s);
+    else if (collision == LBM_KBC) launch_typed<27, LBM_KBC, double>(kind, params, s);
+    else launch_typed<27, LBM_BGK, double>(kind, params, s);
+  }
+}
+
+void launch_init_eq(int Q, int precision, void* pop, const uint8_t* types, int32_t nfluid, const double* rho,
+                    const double* u, cudaStream_t s) {
+  if (nfluid <= 0) return;
+  if (precision == LBM_FP32) {
+    if (Q == 19) init_eq_kernel<19, float><<<nfluid, 512, 0, s>>>((float*)pop, types, rho, u);
+    else init_eq_kernel<27, float><<<nfluid, 512, 0, s>>>((float*)pop, types, rho, u);
+  } else {
+    if (Q == 19) init_eq_kernel<19, double><<<nfluid, 512, 0, s>>>((double*)pop, types, rho, u);
+    else init_eq_kernel<27, double><<<nfluid, 512, 0, s>>>((double*)pop, types, rho, u);
+  }
+}
+
+void launch_macroscopic(int Q, int precision, const void* pop, const uint8_t* types, int32_t nfluid, double* rho,
+                        double* u, double* block_mass, cudaStream_t s) {
+  if (nfluid <= 0) return;
+  if (precision == LBM_FP32) {
+    if (Q == 19) macroscopic_kernel<19, float><<<nfluid, 512, 0, s>>>((const float*)pop, types, rho, u, block_mass);
+    else macroscopic_kernel<27, float><<<nfluid, 512, 0, s>>>((const float*)pop, types, rho, u, block_mass);
+  } else {
+    if (Q == 19) macroscopic_kernel<19, double><<<nfluid, 512, 0, s>>>((const double*)pop, types, rho, u, block_mass);
+    else macroscopic_kernel<27, double><<<nfluid, 512, 0, s>>>((const double*)pop, types, rho, u, block_mass);
+  }
+}
+
+}  // namespace lbmr

@@ -1,0 +1,222 @@
+"""Thin ctypes binding of liblbmr.so (include/lbmr.h).
+
+Argument marshalling only: every step of the hot path runs in the library's
+sm_100a kernels.  There is no CPU fallback: if the library is missing, or no
+CUDA device is present when a grid is created, the call raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from typing import Optional, Sequence
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "_lib", "liblbmr.so")
+
+LBM_OK = 0
+STATUS = {0: "LBM_OK", 1: "LBM_E_INVAL", 2: "LBM_E_TILING", 3: "LBM_E_UNBALANCED", 4: "LBM_E_OOM",
+          5: "LBM_E_CUDA", 6: "LBM_E_COMM", 7: "LBM_E_STATE", 8: "LBM_E_UNSUPPORTED"}
+D3Q19, D3Q27 = 19, 27
+BGK, KBC = 0, 1
+FP32, FP64 = 0, 1
+BC_NOSLIP, BC_VELOCITY, BC_OUTFLOW = 0, 1, 2
+
+
+class LBMError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class GridDesc(ctypes.Structure):
+    _fields_ = [
+        ("nx", ctypes.c_int32), ("ny", ctypes.c_int32), ("nz", ctypes.c_int32),
+        ("periodic", ctypes.c_int32 * 3),
+        ("face_bc", ctypes.c_uint8 * 6), ("pad_", ctypes.c_uint8 * 2),
+        ("lattice", ctypes.c_int32), ("collision", ctypes.c_int32), ("precision", ctypes.c_int32),
+        ("omega0", ctypes.c_double),
+        ("n_ranks", ctypes.c_int32), ("rank", ctypes.c_int32),
+        ("stream", ctypes.c_void_p),
+    ]
+
+
+class GridInfo(ctypes.Structure):
+    _fields_ = [
+        ("levels", ctypes.c_int32), ("Q", ctypes.c_int32), ("precision", ctypes.c_int32),
+        ("kernels_per_step", ctypes.c_int32),
+        ("leaves", ctypes.c_int64 * 16), ("blocks", ctypes.c_int64 * 16),
+        ("special_blocks", ctypes.c_int64 * 16), ("special_cells", ctypes.c_int64 * 16),
+        ("total_blocks", ctypes.c_int64 * 16),
+        ("device_bytes", ctypes.c_int64), ("steps_done", ctypes.c_int64),
+    ]
+
+
+EXPORTS = ["lbm_grid_create", "lbm_set_bc", "lbm_init_equilibrium", "lbm_init_uniform", "lbm_step",
+           "lbm_macroscopic", "lbm_stats", "lbm_grid_get_info", "lbm_profile_levels", "lbm_synchronize",
+           "lbm_grid_destroy", "lbm_last_error", "lbm_version"]
+
+_lib = None
+
+
+def load_library(path: str = LIB_PATH):
+    """Load liblbmr.so; raises if it is missing (no fallback)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(path):
+        raise ImportError(f"liblbmr.so not built ({path}); run __graft_entry__.build()")
+    lib = ctypes.CDLL(path)
+    P = ctypes.c_void_p
+    dp = ctypes.POINTER(ctypes.c_double)
+    lp = ctypes.POINTER(ctypes.c_int64)
+    lib.lbm_grid_create.argtypes = [ctypes.POINTER(GridDesc), ctypes.c_int32, ctypes.POINTER(ctypes.c_void_p),
+                                    ctypes.POINTER(P)]
+    lib.lbm_set_bc.argtypes = [P, ctypes.c_int32, ctypes.c_int32, dp]
+    lib.lbm_init_equilibrium.argtypes = [P, ctypes.c_int32, dp, dp]
+    lib.lbm_init_uniform.argtypes = [P, ctypes.c_double, dp]
+    lib.lbm_step.argtypes = [P, ctypes.c_int32]
+    lib.lbm_macroscopic.argtypes = [P, ctypes.c_int32, dp, dp]
+    lib.lbm_stats.argtypes = [P, lp, dp]
+    lib.lbm_grid_get_info.argtypes = [P, ctypes.POINTER(GridInfo)]
+    lib.lbm_profile_levels.argtypes = [P, ctypes.c_int32, dp, lp]
+    lib.lbm_synchronize.argtypes = [P]
+    lib.lbm_grid_destroy.argtypes = [P]
+    lib.lbm_grid_destroy.restype = None
+    lib.lbm_last_error.restype = ctypes.c_char_p
+    lib.lbm_version.restype = ctypes.c_char_p
+    for name in EXPORTS:
+        f = getattr(lib, name)
+        if f.restype is ctypes.c_int:
+            f.restype = ctypes.c_int
+    _lib = lib
+    return lib
+
+
+def _check(st: int):
+    if st != LBM_OK:
+        raise LBMError(st, _lib.lbm_last_error().decode())
+
+
+def _dp(a: Optional[np.ndarray]):
+    if a is None:
+        return None
+    return a.ctypes.data_as(ctypes.POINTER(ctypes.c_double))
+
+
+class Grid:
+    """A multi-level LBM grid on the current CUDA device (one per rank)."""
+
+    def __init__(self, nx: int, ny: int, nz: int, masks: Sequence[np.ndarray], *, periodic=(0, 0, 0),
+                 face_bc=(0, 0, 0, 0, 0, 0), lattice: int = D3Q19, collision: int = BGK,
+                 precision: int = FP32, omega0: float = 1.0, stream: Optional[int] = None):
+        lib = load_library()
+        self.lib = lib
+        self.shape0 = (nx, ny, nz)
+        self.levels = len(masks)
+        self._masks = [np.ascontiguousarray(m, dtype=np.uint8) for m in masks]
+        for L, m in enumerate(self._masks):
+            if m.shape != (nx << L, ny << L, nz << L):
+                raise ValueError(f"mask {L} has shape {m.shape}, expected {(nx << L, ny << L, nz << L)}")
+        d = GridDesc()
+        d.nx, d.ny, d.nz = nx, ny, nz
+        for a in range(3):
+            d.periodic[a] = int(periodic[a])
+        for f in range(6):
+            d.face_bc[f] = int(face_bc[f])
+        d.lattice, d.collision, d.precision = int(lattice), int(collision), int(precision)
+        d.omega0 = float(omega0)
+        d.n_ranks, d.rank = 1, 0
+        d.stream = stream
+        ptrs = (ctypes.c_void_p * self.levels)(*[m.ctypes.data for m in self._masks])
+        h = ctypes.c_void_p()
+        _check(lib.lbm_grid_create(ctypes.byref(d), self.levels, ptrs, ctypes.byref(h)))
+        self.h = h
+        self._masks = None  # the library copied what it needs
+
+    # -- lifecycle -------------------------------------------------------
+    def close(self):
+        if getattr(self, "h", None) is not None and self.h.value:
+            self.lib.lbm_grid_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    # -- API -----------------------------------------------------------------
+    def set_bc(self, cls: int, kind: int, u=(0.0, 0.0, 0.0)):
+        u = np.ascontiguousarray(u, dtype=np.float64)
+        _check(self.lib.lbm_set_bc(self.h, int(cls), int(kind), _dp(u)))
+
+    def level_shape(self, L: int):
+        nx, ny, nz = self.shape0
+        return (nx << L, ny << L, nz << L)
+
+    def init_equilibrium(self, L: int, rho: Optional[np.ndarray] = None, u: Optional[np.ndarray] = None):
+        shape = self.level_shape(L)
+        r = None if rho is None else np.ascontiguousarray(rho, dtype=np.float64).reshape(shape)
+        v = None if u is None else np.ascontiguousarray(u, dtype=np.float64).reshape(shape + (3,))
+        _check(self.lib.lbm_init_equilibrium(self.h, int(L), _dp(r), _dp(v)))
+
+    def init_uniform(self, rho0: float = 1.0, u0=(0.0, 0.0, 0.0)):
+        u = np.ascontiguousarray(u0, dtype=np.float64)
+        _check(self.lib.lbm_init_uniform(self.h, float(rho0), _dp(u)))
+
+    def step(self, n_coarse: int = 1):
+        _check(self.lib.lbm_step(self.h, int(n_coarse)))
+
+    def synchronize(self):
+        _check(self.lib.lbm_synchronize(self.h))
+
+    def macroscopic(self, L: int):
+        shape = self.level_shape(L)
+        rho = np.empty(shape)
+        u = np.empty(shape + (3,))
+        _check(self.lib.lbm_macroscopic(self.h, int(L), _dp(rho), _dp(u)))
+        return rho, u
+
+    def stats(self):
+        leaves = np.zeros(self.levels, dtype=np.int64)
+        mass = ctypes.c_double()
+        _check(self.lib.lbm_stats(self.h, leaves.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)),
+                                  ctypes.byref(mass)))
+        return leaves, mass.value
+
+    def info(self) -> GridInfo:
+        gi = GridInfo()
+        _check(self.lib.lbm_grid_get_info(self.h, ctypes.byref(gi)))
+        return gi
+
+    def profile_levels(self, n_coarse: int):
+        ms = np.zeros(self.levels)
+        cnt = np.zeros(self.levels, dtype=np.int64)
+        _check(self.lib.lbm_profile_levels(self.h, int(n_coarse), _dp(ms),
+                                           cnt.ctypes.data_as(ctypes.POINTER(ctypes.c_int64))))
+        return ms, cnt
+
+
+def grid_from_problem(prob, precision: int = FP32, stream: Optional[int] = None, init: bool = True) -> Grid:
+    """Build a Grid from an ``lbm_inputs.Problem`` (masks, BCs, initial state)."""
+    g = Grid(prob.nx, prob.ny, prob.nz, prob.masks, periodic=prob.periodic, face_bc=prob.face_bc,
+             lattice=prob.Q, collision=KBC if prob.collision == "kbc" else BGK, precision=precision,
+             omega0=prob.omega0, stream=stream)
+    for cls, (kind, u) in prob.bc.items():
+        g.set_bc(cls, kind, u)
+    if init:
+        if prob.init_rho is None and prob.init_u is None:
+            g.init_uniform(prob.uniform_rho, prob.uniform_u)
+        else:
+            for L in range(prob.levels):
+                rho, u = prob.init_fields(L)
+                g.init_equilibrium(L, rho, u)
+    return g

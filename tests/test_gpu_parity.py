@@ -1,0 +1,135 @@
+"""GPU (liblbmr.so, sm_100a) vs fp64 oracle parity, element by element on ρ, u
+of every fluid leaf of every level.  Bars (north_star): fp32 ≤ 1e-5,
+fp64 ≤ 1e-12 (max error normalised by the field maximum)."""
+import numpy as np
+import pytest
+
+import lbm_inputs as I
+from tests._parity import TOL, errors, gpu_run, oracle_run
+
+pytestmark = pytest.mark.gpu
+
+FP32, FP64 = 0, 1
+
+_cache = {}
+
+
+def _oracle(key, prob, steps):
+    if key not in _cache:
+        _cache[key] = oracle_run(prob, steps)
+    return _cache[key]
+
+
+def check(prob, steps, prec, key=None, chunks=None):
+    ora = _oracle(key or (prob.name, steps), prob, steps)
+    er, eu = errors(gpu_run(prob, steps, prec, chunks=chunks), ora)
+    assert er <= TOL[prec] and eu <= TOL[prec], (prob.name, prec, er, eu)
+    return er, eu
+
+
+@pytest.mark.parametrize("prec", [FP64, FP32])
+@pytest.mark.parametrize("steps", [20, 100])
+def test_cfg1_cavity2(prec, steps):
+    """BASELINE configs[0]: D3Q19 BGK cavity 32^3, 2 levels, refined core."""
+    check(I.cavity2(), steps, prec)
+
+
+@pytest.mark.parametrize("prec", [FP64, FP32])
+def test_cfg1_cavity2_random_state(prec):
+    check(I.cavity2("r"), 20, prec)
+
+
+def test_step_chunking_is_irrelevant():
+    """lbm_step(a) + lbm_step(b) == lbm_step(a+b) (both graph parities)."""
+    check(I.cavity2("r"), 7, FP64, chunks=[1, 2, 3, 1])
+
+
+RANDOM = [
+    dict(seed=31, n=(12, 10, 9), levels=3),
+    dict(seed=32, n=(12, 10, 9), levels=2, periodic=(1, 1, 1), p_bc=0.0),
+    dict(seed=33, n=(9, 11, 10), levels=4, p_refine=0.5),
+    dict(seed=34, n=(10, 10, 10), levels=3, Q=27),
+    dict(seed=35, n=(10, 10, 10), levels=3, Q=27, collision="kbc"),
+    dict(seed=36, n=(13, 9, 11), levels=3, periodic=(0, 0, 0), p_bc=0.15),
+    dict(seed=37, n=(16, 8, 8), levels=3, periodic=(1, 0, 1)),
+]
+
+
+@pytest.mark.parametrize("prec", [FP64, FP32])
+@pytest.mark.parametrize("case", RANDOM, ids=lambda c: f"s{c['seed']}")
+def test_random_balanced_grids(case, prec):
+    """Random strong-2:1 grids with random BC leaves, ragged (non multiple of
+    8) dimensions, periodic/non-periodic mixes, 2-4 levels."""
+    kw = dict(p_refine=0.6)
+    kw.update(case)
+    check(I.random_balanced(**kw), 6, prec, key=("random", case["seed"]))
+
+
+@pytest.mark.parametrize("prec", [FP64, FP32])
+def test_single_level_ragged_periodic(prec):
+    """Single level, periodic, 13x9x11: wrap-around through partial blocks."""
+    p = I.uniform(n=8, omega=1.6)
+    p.nx, p.ny, p.nz = 13, 9, 11
+    p.masks = [np.ones((13, 9, 11), dtype=np.uint8)]
+    rng = np.random.default_rng(5)
+    p.init_rho = [1 + 0.01 * rng.uniform(-1, 1, (13, 9, 11))]
+    p.init_u = [0.03 * rng.uniform(-1, 1, (13, 9, 11, 3))]
+    check(p, 10, prec, key="ragged")
+
+
+@pytest.mark.parametrize("prec", [FP64, FP32])
+def test_cfg3_sphere_reduced(prec):
+    """cfg3 geometry at 1/4 scale (64x32x32 coarse, 3 levels, sphere BC
+    leaves, inlet / outflow / walls)."""
+    check(I.sphere3(scale=4), 20, prec)
+
+
+@pytest.mark.parametrize("prec", [FP64, FP32])
+def test_cfg4_kbc_mini(prec):
+    """cfg4 type: D3Q27 KBC cavity, 4 wall-refined levels (16^3 coarse)."""
+    check(I.cavity4_kbc("mini"), 6, prec)
+
+
+@pytest.mark.parametrize("prec", [FP64, FP32])
+def test_cfg5_tunnel_reduced(prec):
+    """cfg5 geometry at 1/5 scale (40x21x21 coarse, 4 levels)."""
+    check(I.tunnel4(scale=5), 4, prec)
+
+
+@pytest.mark.parametrize("prec", [FP64, FP32])
+def test_uniform_equilibrium_invariance(prec):
+    """T7 on the GPU: a uniform equilibrium stays uniform through every
+    interface (corners included) to rounding."""
+    p = I.refined_box(levels=3, n=(16, 16, 16))
+    p.uniform_rho, p.uniform_u = 1.02, (0.031, -0.017, 0.022)
+    from paper_conf_ipps_mahmoudsm24_b200 import lbmr
+    g = lbmr.grid_from_problem(p, precision=prec)
+    g.step(5)
+    tol = 1e-14 if prec == FP64 else 2e-7
+    for L in range(p.levels):
+        r, u = g.macroscopic(L)
+        m = ~np.isnan(r)
+        assert np.abs(r[m] - 1.02).max() < tol
+        assert np.abs(u[m] - np.array(p.uniform_u)).max() < tol
+
+
+def test_couette_gpu_exact():
+    """T9 on the GPU: refined wall layers, steady linear profile exact (fp64)."""
+    H, U = 16, 0.02
+    p = I.couette(levels=3, H=H, n_xz=8, U=U, omega0=1.0)
+    p.init_u = []
+    for L in range(3):
+        sh = p.level_shape(L)
+        y = (np.arange(sh[1]) + 0.5) / (1 << L)
+        u = np.zeros(sh + (3,))
+        u[..., 0] = (U * y / H)[None, :, None]
+        p.init_u.append(u)
+    from paper_conf_ipps_mahmoudsm24_b200 import lbmr
+    g = lbmr.grid_from_problem(p, precision=FP64)
+    g.step(1500)
+    for L in range(3):
+        r, u = g.macroscopic(L)
+        sh = p.level_shape(L)
+        y = (np.arange(sh[1]) + 0.5) / (1 << L)
+        m = ~np.isnan(r)
+        assert np.abs(u[..., 0] - (U * y / H)[None, :, None])[m].max() / U < 1e-12
