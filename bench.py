@@ -1,0 +1,305 @@
+#!/usr/bin/env python
+"""Benchmark: MLUPS (fine-equivalent) of the multi-level LBM coarse step on B200.
+
+Default workload: BASELINE configs[4] / SURVEY cfg5 "tunnel4" — D3Q19 BGK,
+4 levels, 200x105x105 coarse = 1600x840x840 finest-equivalent, fp32 (shifted
+populations), the configuration the metric's 1/2/4/8-GPU target is quoted on
+(it fits one B200: 7.3 GB of populations).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                  [--config tunnel4|sphere3|cavity4_kbc|uniform512|cavity2]
+
+MLUPS = sum_L V_L 2^L K / T[us] (reading R-A13), V_L = fluid leaves of
+level L.  T is measured with CUDA events on the grid's stream around K graph
+replays (inputs resident in HBM; the 7.3 GB working set exceeds the 126 MB L2,
+so no flush is needed), max over ranks.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import lbm_inputs as I  # noqa: E402
+
+METRIC = "MLUPS (fine-equivalent) per step at 1/2/4/8 B200 and % of HBM roofline"
+
+CONFIGS = {
+    "tunnel4": (lambda: I.tunnel4(), "cfg5 tunnel4: D3Q19 BGK, 4 levels, 200x105x105 coarse (1600x840x840 eff.)"),
+    "sphere3": (lambda: I.sphere3(), "cfg3 sphere3: D3Q19 BGK, 3 levels, 256x128x128 coarse, Re=3700"),
+    "cavity4_kbc": (lambda: I.cavity4_kbc(), "cfg4 cavity4: D3Q27 KBC, 4 levels, 384^3 effective"),
+    "uniform512": (lambda: I.uniform(512), "cfg2 uniform512: D3Q19 BGK, single level 512^3 periodic"),
+    "cavity2": (lambda: I.cavity2(), "cfg1 cavity2: D3Q19 BGK, 2 levels, 32^3 coarse"),
+}
+# bounded oracle sample for --impl reference (one coarse step per timed step)
+REF_SAMPLE = {
+    "tunnel4": (lambda: I.tunnel4(scale=5), "tunnel4 geometry at 1/5 scale (40x21x21 coarse, 4 levels)"),
+    "sphere3": (lambda: I.sphere3(scale=4), "sphere3 geometry at 1/4 scale (64x32x32 coarse, 3 levels)"),
+    "cavity4_kbc": (lambda: I.cavity4_kbc("mini"), "cavity4 KBC at 16^3 coarse, 4 levels"),
+    "uniform512": (lambda: I.uniform(64), "uniform periodic 64^3"),
+    "cavity2": (lambda: I.cavity2(), "cavity2 (full size)"),
+}
+
+
+def updates_per_step(leaves):
+    return sum(int(v) << L for L, v in enumerate(leaves))
+
+
+def peak_hbm():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device_index: int):
+        self.proc = None
+        self.dev = device_index
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.dev), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "50"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+        time.sleep(0.3)
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.1)
+        self.proc.terminate()
+        out, _ = self.proc.communicate(timeout=10)
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in out.strip().splitlines():
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) < 7:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx = float(parts[1])
+            except ValueError:
+                continue
+            for n, v in zip(names, parts[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        load = [s for s in sm if mx and s > 0.5 * mx] or sm
+        return {"sm_mhz": statistics.median(load) if load else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def dist_setup():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def run_reference(args, ws, rank):
+    """The oracle (fp64 CPU) as it stands, timed on the host cores."""
+    import oracle
+    if rank != 0:
+        return
+    build_fn, sample = REF_SAMPLE[args.config]
+    prob = build_fn()
+    o = oracle.Oracle(prob)
+    upd = updates_per_step(prob.fluid_leaves())
+    for _ in range(args.warmup):
+        o.step(1)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        o.step(1)
+    dt = time.perf_counter() - t0
+    value = upd * args.steps / (dt * 1e6)
+    cores = len(os.sched_getaffinity(0))
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "MLUPS", "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3 / args.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic", "config": {"workload": CONFIGS[args.config][1], "sample": sample},
+        "cpu_baseline": {"value": value, "unit": "MLUPS", "cores": cores, "kind": "oracle",
+                         "sample": f"{sample}; one oracle coarse step per timed step"},
+        "e2e": {"value": value, "unit": "MLUPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def cpu_baseline(prob):
+    """Oracle (as it stands) on the same workload, one coarse step, host cores."""
+    import oracle
+    o = oracle.Oracle(prob)
+    t0 = time.perf_counter()
+    o.step(1)
+    dt = time.perf_counter() - t0
+    del o
+    upd = updates_per_step(prob.fluid_leaves())
+    return {"value": upd / (dt * 1e6), "unit": "MLUPS", "cores": len(os.sched_getaffinity(0)), "kind": "oracle",
+            "sample": "one coarse step of the same workload (fp64 C++ OpenMP oracle, literal Alg.1)",
+            "seconds": dt}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=100)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="tunnel4", choices=sorted(CONFIGS))
+    ap.add_argument("--precision", default="fp32", choices=["fp32", "fp64"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--profile-steps", type=int, default=10)
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    ws, rank, local = dist_setup()
+
+    if args.impl == "reference":
+        run_reference(args, ws, rank)
+        return
+
+    import torch
+    torch.cuda.set_device(local)
+    if ws > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    from paper_conf_ipps_mahmoudsm24_b200 import lbmr
+
+    build_fn, desc = CONFIGS[args.config]
+    prob = build_fn()
+    prec = lbmr.FP32 if args.precision == "fp32" else lbmr.FP64
+    stream = torch.cuda.Stream()
+    t0 = time.perf_counter()
+    g = lbmr.grid_from_problem(prob, precision=prec, stream=stream.cuda_stream, init=False)
+    g.init_uniform(prob.uniform_rho, prob.uniform_u) if prob.init_u is None else [
+        g.init_equilibrium(L, *prob.init_fields(L)) for L in range(prob.levels)]
+    setup_s = time.perf_counter() - t0
+    info = g.info()
+    leaves = [int(info.leaves[L]) for L in range(prob.levels)]
+    upd = updates_per_step(leaves)
+    kernels_per_step = int(info.kernels_per_step)
+
+    g.step(args.warmup)
+    g.synchronize()
+
+    def barrier():
+        if ws > 1:
+            torch.distributed.barrier()
+
+    sampler = ClockSampler(local)
+    sampler.start()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    barrier()
+    torch.cuda.synchronize()
+    ev0.record(stream)
+    g.step(args.steps)
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    barrier()
+    clocks = sampler.stop()
+    ms = ev0.elapsed_time(ev1)
+    if ws > 1:
+        t = torch.tensor([ms], device="cuda", dtype=torch.float64)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        ms = float(t.item())
+    value = upd * args.steps * ws / (ms * 1e3)
+
+    # per-level device time (instrumented launches, CUDA events on the same stream)
+    ms_lvl, cnt_lvl = g.profile_levels(args.profile_steps)
+    tsz = 4 if prec == lbmr.FP32 else 8
+    bpu = 2 * prob.Q * tsz
+    dom = int(np.argmax(ms_lvl))
+    per_launch_ms = ms_lvl[dom] / max(cnt_lvl[dom], 1)
+    achieved = leaves[dom] * bpu / (per_launch_ms * 1e-3) / 1e9
+    peak, peak_src = peak_hbm()
+    per_level = []
+    for L in range(prob.levels):
+        pl = ms_lvl[L] / max(cnt_lvl[L], 1)
+        gbs = leaves[L] * bpu / (pl * 1e-3) / 1e9 if pl > 0 else None
+        per_level.append({"level": L, "leaves": leaves[L], "launches": int(cnt_lvl[L]), "ms_per_launch": pl,
+                          "GBs": gbs, "frac": gbs / peak if gbs else None,
+                          "share_of_step": ms_lvl[L] / max(ms_lvl.sum(), 1e-12)})
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tpath):
+        try:
+            tj = json.load(open(tpath)).get(f"{args.config}_{args.precision}")
+            if tj:
+                traffic = tj.get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+
+    # e2e through the public API with host buffers: per step an H2D BC update
+    # (inlet velocity) and a D2H read of the step's diagnostic (total mass)
+    n_e2e = min(args.steps, 20)
+    u_in = prob.bc.get(I.CLS_LID, (1, (0.0, 0.0, 0.0)))[1]
+    torch.cuda.synchronize()
+    barrier()
+    t0 = time.perf_counter()
+    for _ in range(n_e2e):
+        g.set_bc(I.CLS_LID, lbmr.BC_VELOCITY, u_in)
+        g.step(1)
+        _, mass = g.stats()
+    e2e_s = time.perf_counter() - t0
+    if ws > 1:
+        t = torch.tensor([e2e_s], device="cuda", dtype=torch.float64)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        e2e_s = float(t.item())
+    e2e = {"value": upd * n_e2e * ws / (e2e_s * 1e6), "unit": "MLUPS",
+           "h2d_bytes_per_step": 32 + 27,
+           "d2h_bytes_per_step": 8 * int(sum(info.blocks[L] for L in range(prob.levels))),
+           "steps": n_e2e, "what": "per step: lbm_set_bc (H2D) + lbm_step(1) + lbm_stats mass (D2H), wall clock"}
+
+    gi = g.info()
+    dev_bytes = int(gi.device_bytes)
+    g.close()
+    cpu = None
+    if rank == 0 and ws == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(prob)
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "MLUPS", "n_gpus": ws, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+            "scaling": "weak" if ws > 1 else "strong", "vs_baseline": None,
+            "dtype": "f32" if prec == lbmr.FP32 else "f64", "data": "synthetic",
+            "config": {"workload": desc, "levels": prob.levels, "leaves": leaves, "updates_per_step": upd,
+                       "parallelism": "replicas" if ws > 1 else "single",
+                       "l2": f"working set {dev_bytes / 1e9:.2f} GB > 126 MB L2 (no flush needed)",
+                       "precision": args.precision, "setup_s": round(setup_s, 2)},
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic, "kernel": f"level_step L{dom}",
+                         "bytes_per_update": bpu, "peak_source": peak_src,
+                         "step_frac": value * 1e6 / ws * bpu / 1e9 / peak},
+            "per_level": per_level,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": kernels_per_step * args.steps,
+            "clocks": clocks,
+        }
+        print(json.dumps(line), flush=True)
+    if ws > 1:
+        torch.distributed.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

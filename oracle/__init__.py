@@ -57,6 +57,7 @@ def _load():
         lib.ora_num_leaves.argtypes = [P, ctypes.c_int]
         lib.ora_num_leaves.restype = ctypes.c_int64
         lib.ora_init_equilibrium.argtypes = [P, ctypes.c_int, dp, dp]
+        lib.ora_init_uniform.argtypes = [P, ctypes.c_double, dp]
         lib.ora_step.argtypes = [P, ctypes.c_int]
         lib.ora_macroscopic.argtypes = [P, ctypes.c_int, dp, dp]
         lib.ora_get_f.argtypes = [P, ctypes.c_int, dp]
@@ -121,9 +122,13 @@ class Oracle:
             raise ValueError("oracle: " + err.value.decode())
         self.h = ctypes.c_void_p(h)
         if init:
-            for L in range(prob.levels):
-                rho, uu = prob.init_fields(L)
-                self.init_equilibrium(L, rho, uu)
+            if prob.init_rho is None and prob.init_u is None:
+                u0 = np.ascontiguousarray(prob.uniform_u, dtype=np.float64)
+                lib.ora_init_uniform(self.h, float(prob.uniform_rho), _dp(u0))
+            else:
+                for L in range(prob.levels):
+                    rho, uu = prob.init_fields(L)
+                    self.init_equilibrium(L, rho, uu)
 
     def __del__(self):
         h = getattr(self, "h", None)
