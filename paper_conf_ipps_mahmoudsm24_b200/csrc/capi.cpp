@@ -289,7 +289,15 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     delete g;
     return fail((lbm_status)st, err);
   }
-  for (int L = 0; L < levels; ++L) g->omega.push_back(omega_level(d->omega0, L));
+  for (int L = 0; L < levels; ++L) {
+    g->omega.push_back(omega_level(d->omega0, L));
+    // kernels index populations with 32-bit offsets
+    if ((uint64_t)g->host[L].nblocks * (uint64_t)g->Q * kCells >= (1ull << 32)) {
+      delete g;
+      return fail(LBM_E_UNSUPPORTED, "level " + std::to_string(L) +
+                                         " too large for one device (> 2^32 populations); use more ranks");
+    }
+  }
 
   auto cleanup = [&](lbm_status s) {
     std::string keep = g_err;

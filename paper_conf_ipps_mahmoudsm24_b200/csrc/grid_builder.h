@@ -20,7 +20,7 @@ struct HostLevel {
   std::vector<int32_t> blkmap;   // [nb0*nb1*nb2] block id or -1; index (bx*nb1+by)*nb2+bz
   std::vector<int32_t> origin;   // [nblocks*3] block coordinates
   std::vector<uint8_t> types;    // [nblocks*512] cell type (lattice.h codes), local = x+8y+64z
-  std::vector<int32_t> nbr;      // [nfluid*27] neighbour block ids (-1 none)
+  std::vector<int32_t> nbr;      // [nfluid*kRec] block records (lattice.h: neighbours, slot, origin)
   std::vector<int32_t> special_slot;  // [nfluid] index into cellinfo or -1 (plain block)
   std::vector<uint32_t> cellinfo;     // [nspecial*512] bit q: slow link q; bit31: fluid leaf
 };

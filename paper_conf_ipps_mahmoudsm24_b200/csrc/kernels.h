@@ -27,7 +27,7 @@ struct BCEntry {
 template <typename T>
 struct StepParams {
   LevelView own, coarse, fine;
-  const int32_t* nbr;           // [nfluid][27]
+  const int32_t* nbr;           // [nfluid][kRec] block records (lattice.h)
   const int32_t* special_slot;  // [nfluid]
   const uint32_t* cellinfo;     // [nspecial][512]
   const int32_t* origin;        // [nblocks][3] block coordinates

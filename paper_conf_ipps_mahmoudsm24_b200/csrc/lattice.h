@@ -40,6 +40,12 @@ LBM_HD constexpr int nbr_slot(int dx, int dy, int dz) { return (dx + 1) + 3 * (d
 constexpr int kBlock = 8;            // B = 8 (B compile time)
 constexpr int kCells = 512;          // B^3
 constexpr unsigned kFluidBit = 1u << 31;
+// per-fluid-block record of 32 int32 (one 128-byte line, loaded by one warp
+// instruction): [0..26] neighbour block ids by nbr_slot (-1 none), [27]
+// special slot (-1 plain), [28..30] block coordinates, [31] unused
+constexpr int kRec = 32;
+constexpr int kRecSlot = 27;
+constexpr int kRecOrigin = 28;
 
 // cell type codes stored per block (mask codes + derived states)
 constexpr unsigned char kAbsent = 0;    // covered by a coarser leaf, or outside the domain

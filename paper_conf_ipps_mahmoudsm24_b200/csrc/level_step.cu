@@ -21,8 +21,11 @@
 // source is not a same-level fluid leaf reachable by the block arithmetic are
 // flagged per cell by the host builder (cellinfo) and resolved in
 // slow_link(); blocks without such cells (the bulk) never read cellinfo.
+#include <algorithm>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
+#include <utility>
 
 #include "../../include/lbmr.h"
 #include "kernels.h"
@@ -67,18 +70,60 @@ __device__ __forceinline__ T geq(int q, T drho, T rho, T ux, T uy, T uz, T usq15
   return T(weight<Q>(q)) * (drho + rho * (T(3) * eu + T(4.5) * eu * eu - usq15));
 }
 
+template <typename T>
+__device__ __forceinline__ T recip(T x) {
+  return T(1) / x;
+}
+template <>
+__device__ __forceinline__ float recip<float>(float x) {
+  return __frcp_rn(x);  // correctly rounded, no division sequence
+}
+
+// weight class of direction q: 0 rest, 1 axis, 2 edge, 3 corner
+__host__ __device__ constexpr int wclass(int q) { return q == 0 ? 0 : q < 7 ? 1 : q < 19 ? 2 : 3; }
+
+// BGK, Eq.(3) with Eq.(5), on shifted populations, organised by opposite
+// pairs (q, q+1):  ω g^eq_q = A_w + B_w (e_q.j) + C_w (e_q.j)^2 with
+//   A_w = ω w (δρ - 1.5 |j|^2/ρ),  B_w = 3 ω w,  C_w = 4.5 ω w / ρ
+// (ρ u = j), so the pair shares A + C (e.j)^2 and flips the sign of B (e.j).
 template <int Q, typename T>
 __device__ __forceinline__ void collide_bgk(T (&g)[Q], T omega) {
-  T drho, jx, jy, jz;
-  moments<Q, T>(g, drho, jx, jy, jz);
-  const T rho = T(1) + drho;
-  const T inv = T(1) / rho;
-  const T ux = jx * inv, uy = jy * inv, uz = jz * inv;
-  const T usq15 = T(1.5) * (ux * ux + uy * uy + uz * uz);
+  T drho = g[0], jx = T(0), jy = T(0), jz = T(0);
 #pragma unroll
-  for (int q = 0; q < Q; ++q) {
-    const T e = geq<Q, T>(q, drho, rho, ux, uy, uz, usq15);
-    g[q] = g[q] - omega * (g[q] - e);
+  for (int q = 1; q < Q; q += 2) {
+    const T s = g[q] + g[q + 1];
+    const T d = g[q] - g[q + 1];
+    drho += s;
+    if (ex(q) > 0) jx += d; else if (ex(q) < 0) jx -= d;
+    if (ey(q) > 0) jy += d; else if (ey(q) < 0) jy -= d;
+    if (ez(q) > 0) jz += d; else if (ez(q) < 0) jz -= d;
+  }
+  const T inv = recip<T>(T(1) + drho);
+  const T jj = jx * jx + jy * jy + jz * jz;
+  const T base = omega * (drho - T(1.5) * jj * inv);
+  const T cfac = T(4.5) * omega * inv;
+  const T bfac = T(3) * omega;
+  const T omw = T(1) - omega;
+  T A[4], B[4], C[4];
+#pragma unroll
+  for (int c = 0; c < 4; ++c) {
+    const T w = T(weight<Q>(c == 0 ? 0 : c == 1 ? 1 : c == 2 ? 7 : 19));
+    A[c] = w * base;
+    B[c] = w * bfac;
+    C[c] = w * cfac;
+  }
+  g[0] = omw * g[0] + A[0];
+#pragma unroll
+  for (int q = 1; q < Q; q += 2) {
+    T ej = T(0);
+    if (ex(q) > 0) ej += jx; else if (ex(q) < 0) ej -= jx;
+    if (ey(q) > 0) ej += jy; else if (ey(q) < 0) ej -= jy;
+    if (ez(q) > 0) ej += jz; else if (ez(q) < 0) ej -= jz;
+    const int c = wclass(q);
+    const T sym = C[c] * ej * ej + A[c];
+    const T asym = B[c] * ej;
+    g[q] = omw * g[q] + (sym + asym);
+    g[q + 1] = omw * g[q + 1] + (sym - asym);
   }
 }
 
@@ -244,50 +289,125 @@ __device__ __forceinline__ T slow_link(const StepParams<T>& P, int q, int blk, i
 }
 
 // ---------------------------------------------------------------- fused kernel
-template <int Q, int COLL, typename T, bool STREAM>
-__global__ void __launch_bounds__(256) level_step_kernel(const StepParams<T> P) {
-  __shared__ int s_nbr[27];
-  const int blk = blockIdx.x >> 1;
-  const int t = ((blockIdx.x & 1) << 8) | threadIdx.x;
-  if (STREAM && threadIdx.x < 27) s_nbr[threadIdx.x] = __ldg(P.nbr + (size_t)blk * 27 + threadIdx.x);
-  const int slot = __ldg(P.special_slot + blk);
-  uint32_t info = kFluidBit;
-  if (slot >= 0) info = __ldg(P.cellinfo + (size_t)slot * kCells + t);
-  if (STREAM) __syncthreads();
-  if (!(info & kFluidBit)) return;
+// Per-thread source geometry of the same-level pull inside an 8^3 block:
+// the source coordinate along each axis for e = +1 / -1 / 0 and the
+// neighbour-slot offset, nonzero only for a thread on the block face.
+struct PullGeom {
+  int xm, xp, x0, ym, yp, y0, zm, zp, z0;
+  int dxm, dxp, dym, dyp, dzm, dzp;
+  __device__ __forceinline__ explicit PullGeom(int t) {
+    const int lx = t & 7, ly = (t >> 3) & 7, lz = t >> 6;
+    x0 = lx; xm = (lx - 1) & 7; xp = (lx + 1) & 7;
+    y0 = ly << 3; ym = ((ly - 1) & 7) << 3; yp = ((ly + 1) & 7) << 3;
+    z0 = lz << 6; zm = ((lz - 1) & 7) << 6; zp = ((lz + 1) & 7) << 6;
+    dxm = (lx == 0) ? -1 : 0; dxp = (lx == 7) ? 1 : 0;
+    dym = (ly == 0) ? -3 : 0; dyp = (ly == 7) ? 3 : 0;
+    dzm = (lz == 0) ? -9 : 0; dzp = (lz == 7) ? 9 : 0;
+  }
+  template <int q>
+  __device__ __forceinline__ int local() const {
+    return (ex(q) > 0 ? xm : (ex(q) < 0 ? xp : x0)) | (ey(q) > 0 ? ym : (ey(q) < 0 ? yp : y0)) |
+           (ez(q) > 0 ? zm : (ez(q) < 0 ? zp : z0));
+  }
+  template <int q>
+  __device__ __forceinline__ int slot() const {
+    return 13 + (ex(q) > 0 ? dxm : (ex(q) < 0 ? dxp : 0)) + (ey(q) > 0 ? dym : (ey(q) < 0 ? dyp : 0)) +
+           (ez(q) > 0 ? dzm : (ez(q) < 0 ? dzp : 0));
+  }
+};
 
-  const int lx = t & 7, ly = (t >> 3) & 7, lz = t >> 6;
+template <int Q, typename T, bool PRED, int q>
+__device__ __forceinline__ void pull_one(T (&g)[Q], const T* __restrict__ src, const PullGeom& G, int rec, int blk,
+                                         uint32_t need) {
+  constexpr unsigned FULL = 0xffffffffu;
+  const int nb = (q == 0) ? blk : __shfl_sync(FULL, rec, G.slot<q>());
+  const unsigned off = (unsigned)nb * (unsigned)(Q * kCells) + (unsigned)G.local<q>();
+  const T* p = src + q * kCells;  // constant part folds into the load's immediate offset
+  if (PRED) g[q] = (need & (1u << q)) ? __ldg(p + off) : T(0);
+  else g[q] = __ldg(p + off);
+}
+
+template <int Q, typename T, bool PRED, int... qs>
+__device__ __forceinline__ void pull_all(T (&g)[Q], const T* __restrict__ src, const PullGeom& G, int rec, int blk,
+                                         uint32_t need, std::integer_sequence<int, qs...>) {
+  (pull_one<Q, T, PRED, qs>(g, src, G, rec, blk, need), ...);
+}
+
+template <int Q, typename T>
+__device__ __forceinline__ void store_cell(const T (&g)[Q], T* __restrict__ dst, int blk, int t) {
+  T* d = dst + (unsigned)blk * (unsigned)(Q * kCells) + t;
+#pragma unroll
+  for (int q = 0; q < Q; ++q) d[q * kCells] = g[q];
+}
+
+// One cell (blk, t) of F_L^k.  No shared memory and no barrier: each warp
+// loads its block's 128-byte record (27 neighbour ids, special slot, origin)
+// with one coalesced load and picks neighbour ids with __shfl_sync.  Blocks
+// without special cells (the bulk) take a branch-free pull; the branch on the
+// block's slot is warp-uniform.  Offsets are 32-bit (host-checked).
+template <int Q, int COLL, typename T, bool STREAM>
+__device__ __forceinline__ void process_cell(const StepParams<T>& P, int blk, int t) {
+  constexpr unsigned FULL = 0xffffffffu;
+  const int rec = __ldg(P.nbr + blk * kRec + (threadIdx.x & 31));
+  const int slot = __shfl_sync(FULL, rec, kRecSlot);
   T g[Q];
-  if (STREAM) {
+  if (!STREAM) {
+    if (slot >= 0 && !(__ldg(P.cellinfo + (unsigned)slot * kCells + t) & kFluidBit)) return;
 #pragma unroll
-    for (int q = 0; q < Q; ++q) {
-      const int sx = lx - ex(q), sy = ly - ey(q), sz = lz - ez(q);
-      const int nb = s_nbr[nbr_slot(sx >> 3, sy >> 3, sz >> 3)];
-      const int sl = (sx & 7) | ((sy & 7) << 3) | ((sz & 7) << 6);
-      g[q] = (info & (1u << q)) ? T(0) : __ldg(P.src + ((size_t)nb * Q + q) * kCells + sl);
+    for (int q = 0; q < Q; ++q) g[q] = __ldg(P.src + ((unsigned)blk * Q + q) * kCells + t);
+    collide<Q, COLL, T>(g, P.omega);
+    store_cell<Q, T>(g, P.dst, blk, t);
+    return;
+  }
+  const PullGeom G(t);
+  if (slot < 0) {
+    // plain block: every cell is a fluid leaf with only same-level links
+    pull_all<Q, T, false>(g, P.src, G, rec, blk, 0u, std::make_integer_sequence<int, Q>{});
+    collide<Q, COLL, T>(g, P.omega);
+    store_cell<Q, T>(g, P.dst, blk, t);
+    return;
+  }
+  const uint32_t info = __ldg(P.cellinfo + (unsigned)slot * kCells + t);
+  const bool fluid = (info & kFluidBit) != 0;
+  const uint32_t need = fluid ? ~info : 0u;
+  pull_all<Q, T, true>(g, P.src, G, rec, blk, need, std::make_integer_sequence<int, Q>{});
+  if (!fluid) return;
+  uint32_t slow = info & ((1u << Q) - 1u);
+  if (slow) {
+    const int lx = t & 7, ly = (t >> 3) & 7, lz = t >> 6;
+    const int px = __ldg(P.origin + 3 * blk) * kBlock + lx;
+    const int py = __ldg(P.origin + 3 * blk + 1) * kBlock + ly;
+    const int pz = __ldg(P.origin + 3 * blk + 2) * kBlock + lz;
+    while (slow) {
+      const int q = __ffs(slow) - 1;
+      slow &= slow - 1;
+      const T v = slow_link<Q, T>(P, q, blk, t, px, py, pz);
+#pragma unroll
+      for (int qq = 0; qq < Q; ++qq)
+        if (qq == q) g[qq] = v;
     }
-    uint32_t slow = info & ((1u << Q) - 1u);
-    if (slow) {
-      const int px = __ldg(P.origin + 3 * blk) * kBlock + lx;
-      const int py = __ldg(P.origin + 3 * blk + 1) * kBlock + ly;
-      const int pz = __ldg(P.origin + 3 * blk + 2) * kBlock + lz;
-      while (slow) {
-        const int q = __ffs(slow) - 1;
-        slow &= slow - 1;
-        const T v = slow_link<Q, T>(P, q, blk, t, px, py, pz);
-#pragma unroll
-        for (int qq = 0; qq < Q; ++qq)
-          if (qq == q) g[qq] = v;
-      }
-    }
-  } else {
-#pragma unroll
-    for (int q = 0; q < Q; ++q) g[q] = __ldg(P.src + ((size_t)blk * Q + q) * kCells + t);
   }
   collide<Q, COLL, T>(g, P.omega);
-  T* d = P.dst + (size_t)blk * Q * kCells + t;
-#pragma unroll
-  for (int q = 0; q < Q; ++q) d[(size_t)q * kCells] = g[q];
+  store_cell<Q, T>(g, P.dst, blk, t);
+}
+
+template <int Q, typename T>
+struct Occ { static constexpr int value = 1; };
+template <>
+struct Occ<19, float> { static constexpr int value = 4; };
+
+// CTA = half an 8^3 block (256 threads, one cell each).
+template <int Q, int COLL, typename T, bool STREAM>
+__global__ void __launch_bounds__(256, Occ<Q, T>::value) level_step_kernel(const StepParams<T> P) {
+  process_cell<Q, COLL, T, STREAM>(P, blockIdx.x >> 1, ((blockIdx.x & 1) << 8) | threadIdx.x);
+}
+
+// Persistent variant: gridDim.x = resident CTAs; each CTA walks half-blocks.
+template <int Q, int COLL, typename T, bool STREAM>
+__global__ void __launch_bounds__(256, Occ<Q, T>::value) level_step_persistent(const StepParams<T> P) {
+  const int n = 2 * P.nfluid;
+  for (int w = blockIdx.x; w < n; w += gridDim.x)
+    process_cell<Q, COLL, T, STREAM>(P, w >> 1, ((w & 1) << 8) | threadIdx.x);
 }
 
 // ---------------------------------------------------------------- init / macroscopic
@@ -353,11 +473,29 @@ __global__ void __launch_bounds__(512) macroscopic_kernel(const T* pop, const ui
 }
 
 // ---------------------------------------------------------------- dispatch
+static int g_variant = -1;  // 0: one CTA per half block, 1: persistent
+static int g_nsm = 0;
+
 template <int Q, int COLL, typename T>
 static void launch_typed(int kind, const void* params, cudaStream_t s) {
   const StepParams<T>& p = *static_cast<const StepParams<T>*>(params);
   if (p.nfluid <= 0) return;
-  dim3 grid(2 * p.nfluid), block(256);
+  if (g_variant < 0) {
+    const char* v = getenv("LBMR_VARIANT");
+    g_variant = v ? atoi(v) : 0;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&g_nsm, cudaDevAttrMultiProcessorCount, dev);
+  }
+  dim3 block(256);
+  if (g_variant == 1 && kind == 0) {
+    int occ = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, level_step_persistent<Q, COLL, T, true>, 256, 0);
+    int grid = std::min(2 * p.nfluid, std::max(1, occ) * g_nsm);
+    level_step_persistent<Q, COLL, T, true><<<grid, block, 0, s>>>(p);
+    return;
+  }
+  dim3 grid(2 * p.nfluid);
   if (kind == 0) level_step_kernel<Q, COLL, T, true><<<grid, block, 0, s>>>(p);
   else level_step_kernel<Q, COLL, T, false><<<grid, block, 0, s>>>(p);
 }
