@@ -30,8 +30,9 @@ def _stale() -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not _stale():
+def build(force: bool = False, verbose: bool = False, out: str = None, defines=()) -> str:
+    lib = out or LIB
+    if not force and out is None and not _stale():
         return LIB
     os.makedirs(LIBDIR, exist_ok=True)
     objs = []
@@ -39,17 +40,17 @@ def build(force: bool = False, verbose: bool = False) -> str:
         src = os.path.join(CSRC, s)
         obj = os.path.join(LIBDIR, s + ".o")
         cmd = [nvcc(), "-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xcompiler", "-fPIC,-fopenmp,-O3",
-               "-I", os.path.join(HERE, "..", "include"), "-c", src, "-o", obj]
+               "-I", os.path.join(HERE, "..", "include"), *[f"-D{d}" for d in defines], "-c", src, "-o", obj]
         if s.endswith(".cu"):
             cmd += ["-Xptxas", "-v"] if verbose else []
         subprocess.check_call(cmd)
         objs.append(obj)
-    tmp = LIB + ".tmp"
+    tmp = lib + ".tmp"
     subprocess.check_call([nvcc(), "-shared", *ARCH, "-o", tmp, *objs, "-Xcompiler", "-fopenmp", "-lgomp"])
-    os.replace(tmp, LIB)
+    os.replace(tmp, lib)
     for o in objs:
         os.remove(o)
-    return LIB
+    return lib
 
 
 if __name__ == "__main__":

@@ -18,6 +18,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -51,6 +52,10 @@ struct DevLevel {
   int32_t* nbr = nullptr;
   int32_t* special_slot = nullptr;
   uint32_t* cellinfo = nullptr;
+  uint32_t* links = nullptr;
+  uint32_t* coal = nullptr;
+  int32_t* plain_ids = nullptr;
+  int32_t* special_ids = nullptr;
   void* pop[2] = {nullptr, nullptr};
 };
 
@@ -72,6 +77,8 @@ struct lbm_grid {
   uint8_t* face_dev = nullptr;
   cudaStream_t stream = nullptr;
   bool own_stream = false;
+  cudaStream_t side = nullptr;          // special blocks run beside the plain ones
+  cudaEvent_t fork = nullptr, join = nullptr;
   cudaGraphExec_t graph[2] = {nullptr, nullptr};
   bool needs_prologue = true;
   bool init_locked = false;  // a step ran since the last init_uniform
@@ -153,7 +160,9 @@ StepParams<T> make_params(const lbm_grid* g, int L, int64_t k) {
   p.fine = view_of(g, L + 1);
   p.nbr = D.nbr;
   p.special_slot = D.special_slot;
-  p.cellinfo = D.cellinfo;
+  p.cellinfo = reinterpret_cast<const uint2*>(D.cellinfo);
+  p.links = reinterpret_cast<const uint2*>(D.links);
+  p.coal = D.coal;
   p.origin = D.origin;
   p.src = static_cast<const T*>(D.pop[k & 1]);
   p.dst = static_cast<T*>(D.pop[(k + 1) & 1]);
@@ -170,14 +179,38 @@ StepParams<T> make_params(const lbm_grid* g, int L, int64_t k) {
   return p;
 }
 
-void launch_F(lbm_grid* g, int L, int64_t k, int kind) {
-  if (g->prec == LBM_FP32) {
-    StepParams<float> p = make_params<float>(g, L, k);
-    launch_level_step(g->Q, g->coll, g->prec, kind, &p, g->stream);
-  } else {
-    StepParams<double> p = make_params<double>(g, L, k);
-    launch_level_step(g->Q, g->coll, g->prec, kind, &p, g->stream);
+template <typename T>
+void launch_F_typed(lbm_grid* g, int L, int64_t k, int kind) {
+  StepParams<T> p = make_params<T>(g, L, k);
+  if (kind == 1) {  // prologue collision
+    launch_level_step(g->Q, g->coll, g->prec, 1, &p, g->stream);
+    return;
   }
+  const HostLevel& H = g->host[L];
+  static int split = -1;
+  if (split < 0) split = getenv("LBMR_SPLIT") ? atoi(getenv("LBMR_SPLIT")) : 0;
+  if (!split) {  // one launch over all blocks in Morton order
+    launch_level_step(g->Q, g->coll, g->prec, 3, &p, g->stream);
+    return;
+  }
+  // fork: special blocks on the side stream, plain blocks on the main stream
+  if (H.special_ids.size()) {
+    cudaEventRecord(g->fork, g->stream);
+    cudaStreamWaitEvent(g->side, g->fork, 0);
+    p.ids = g->dev[L].special_ids;
+    p.nids = (int32_t)H.special_ids.size();
+    launch_level_step(g->Q, g->coll, g->prec, 2, &p, g->side);
+    cudaEventRecord(g->join, g->side);
+  }
+  p.ids = g->dev[L].plain_ids;
+  p.nids = (int32_t)H.plain_ids.size();
+  launch_level_step(g->Q, g->coll, g->prec, 0, &p, g->stream);
+  if (H.special_ids.size()) cudaStreamWaitEvent(g->stream, g->join, 0);
+}
+
+void launch_F(lbm_grid* g, int L, int64_t k, int kind) {
+  if (g->prec == LBM_FP32) launch_F_typed<float>(g, L, k, kind);
+  else launch_F_typed<double>(g, L, k, kind);
 }
 
 // The pipelined order of one coarse step n (0-based): list of (L, k).
@@ -314,6 +347,10 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     }
     g->own_stream = true;
   }
+  if (cudaStreamCreateWithFlags(&g->side, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaEventCreateWithFlags(&g->fork, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&g->join, cudaEventDisableTiming) != cudaSuccess)
+    return cleanup(fail(LBM_E_CUDA, "stream/event creation failed"));
   g->dev.resize(levels);
   lbm_status s;
   for (int L = 0; L < levels; ++L) {
@@ -325,6 +362,10 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     if ((s = dev_upload(g, &D.nbr, H.nbr))) return cleanup(s);
     if ((s = dev_upload(g, &D.special_slot, H.special_slot))) return cleanup(s);
     if ((s = dev_upload(g, &D.cellinfo, H.cellinfo))) return cleanup(s);
+    if ((s = dev_upload(g, &D.links, H.links))) return cleanup(s);
+    if ((s = dev_upload(g, &D.coal, H.coal))) return cleanup(s);
+    if ((s = dev_upload(g, &D.plain_ids, H.plain_ids))) return cleanup(s);
+    if ((s = dev_upload(g, &D.special_ids, H.special_ids))) return cleanup(s);
     for (int b = 0; b < 2; ++b) {
       if ((s = dev_alloc(g, &D.pop[b], pop_bytes(g, L)))) return cleanup(s);
       if (cudaMemset(D.pop[b], 0, pop_bytes(g, L)) != cudaSuccess) return cleanup(fail(LBM_E_CUDA, "memset"));
@@ -332,6 +373,8 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     // the dense per-level tables are on the device now; keep only counters
     std::vector<int32_t>().swap(H.blkmap);
     std::vector<uint32_t>().swap(H.cellinfo);
+    std::vector<uint32_t>().swap(H.links);
+    std::vector<uint32_t>().swap(H.coal);
     std::vector<int32_t>().swap(H.nbr);
   }
   void* p;
@@ -586,7 +629,11 @@ void lbm_grid_destroy(lbm_grid* g) {
   if (g->stream) cudaStreamSynchronize(g->stream);
   for (int p = 0; p < 2; ++p)
     if (g->graph[p]) cudaGraphExecDestroy(g->graph[p]);
+  if (g->side) cudaStreamSynchronize(g->side);
   for (void* p : g->allocs) cudaFree(p);
+  if (g->fork) cudaEventDestroy(g->fork);
+  if (g->join) cudaEventDestroy(g->join);
+  if (g->side) cudaStreamDestroy(g->side);
   if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
   delete g;
 }

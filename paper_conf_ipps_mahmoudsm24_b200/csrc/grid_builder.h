@@ -22,7 +22,13 @@ struct HostLevel {
   std::vector<uint8_t> types;    // [nblocks*512] cell type (lattice.h codes), local = x+8y+64z
   std::vector<int32_t> nbr;      // [nfluid*kRec] block records (lattice.h: neighbours, slot, origin)
   std::vector<int32_t> special_slot;  // [nfluid] index into cellinfo or -1 (plain block)
-  std::vector<uint32_t> cellinfo;     // [nspecial*512] bit q: slow link q; bit31: fluid leaf
+  std::vector<uint32_t> cellinfo;     // [nspecial*512][2]: {bit q = slow link q, bit31 = fluid leaf;
+                                      //  index of the cell's first slow-link record}
+  std::vector<uint32_t> links;        // [nlinks][2] slow-link records (lattice.h kLink*)
+  std::vector<uint32_t> coal;         // coalescence candidate population indices
+  int64_t nlinks = 0;
+  std::vector<int32_t> plain_ids;     // fluid blocks without special cells (Morton order)
+  std::vector<int32_t> special_ids;   // the others (Morton order)
 };
 
 struct BuildInput {

@@ -29,7 +29,9 @@ struct StepParams {
   LevelView own, coarse, fine;
   const int32_t* nbr;           // [nfluid][kRec] block records (lattice.h)
   const int32_t* special_slot;  // [nfluid]
-  const uint32_t* cellinfo;     // [nspecial][512]
+  const uint2* cellinfo;        // [nspecial][512] {slow-link mask | fluid bit, first link record}
+  const uint2* links;           // slow-link records (lattice.h kLink*)
+  const uint32_t* coal;         // coalescence candidate lists
   const int32_t* origin;        // [nblocks][3] block coordinates
   const T* src;                 // C_L^k            [nfluid][Q][512]
   T* dst;                       // C_L^{k+1}
@@ -41,9 +43,13 @@ struct StepParams {
   int32_t periodic[3];
   const uint8_t* face_cls;      // [27] BC class of an out-of-domain source, by outside pattern
   int32_t nfluid;
+  const int32_t* ids;           // blocks this launch processes (plain or special list)
+  int32_t nids;
 };
 
-// kind: 0 = fused stream+collide, 1 = collide only (prologue C_L^1)
+// kind: 0 = fused stream+collide over the plain blocks in ids, 1 = collide only
+// over all fluid blocks (prologue C_L^1), 2 = fused stream+collide over the
+// special blocks in ids
 void launch_level_step(int Q, int collision, int precision, int kind, const void* params, cudaStream_t s);
 
 // g = f^eq(rho,u) - w on the fluid cells of `nfluid` blocks; rho/u compact

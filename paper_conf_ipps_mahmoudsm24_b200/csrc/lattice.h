@@ -47,6 +47,14 @@ constexpr int kRec = 32;
 constexpr int kRecSlot = 27;
 constexpr int kRecOrigin = 28;
 
+// slow-link record {w0, w1}: tag = w1 >> 28
+//  kLinkSame   w0 = population index at level L (irregular same-level source)
+//  kLinkCoarse w0 = population index at level L-1 (Explosion, Eq.10)
+//  kLinkBC     w0 = BC class of the source leaf
+//  kLinkFace   w0 = outside pattern (ox+1)+3(oy+1)+9(oz+1) -> class via face table
+//  kLinkCoal   w0 = first index in the coalescence list, w1 & 0xf = |B|
+constexpr unsigned kLinkSame = 0, kLinkCoarse = 1, kLinkBC = 2, kLinkFace = 3, kLinkCoal = 4;
+
 // cell type codes stored per block (mask codes + derived states)
 constexpr unsigned char kAbsent = 0;    // covered by a coarser leaf, or outside the domain
 constexpr unsigned char kFluid = 1;

@@ -19,8 +19,9 @@
 //
 // The CTA is half an 8^3 block (256 threads, one cell each).  Links whose
 // source is not a same-level fluid leaf reachable by the block arithmetic are
-// flagged per cell by the host builder (cellinfo) and resolved in
-// slow_link(); blocks without such cells (the bulk) never read cellinfo.
+// flagged per cell by the host builder (cellinfo) and resolved from
+// precomputed link records in resolve_slow(); blocks without such cells (the
+// bulk) never read cellinfo.
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
@@ -189,103 +190,78 @@ __device__ __forceinline__ void collide(T (&g)[Q], T omega) {
 }
 
 // ---------------------------------------------------------------- slow links
-__device__ __forceinline__ int lookup(const LevelView& v, int x, int y, int z, int& local) {
-  local = (x & 7) | ((y & 7) << 3) | ((z & 7) << 6);
-  return __ldg(v.blkmap + ((size_t)(x >> 3) * v.nb[1] + (y >> 3)) * v.nb[2] + (z >> 3));
-}
-
-__device__ __forceinline__ unsigned type_at(const LevelView& v, int b, int local) {
-  return b < 0 ? kAbsent : __ldg(v.types + (size_t)b * kCells + local);
-}
-
-__device__ __forceinline__ bool is_bc(unsigned t) { return t != kAbsent && t != kFluid && t != kRefined; }
-
-// BC rule for pulled link q of the cell (blk, t): halfway bounce-back of the
-// cell's own post-collision opposite population, + 6 w_q rho_w e_q.u_w for a
-// moving wall / inlet, g = 0 (f = w_q) for outflow.
-template <int Q, typename T>
-__device__ __forceinline__ T bc_value(const StepParams<T>& P, unsigned cls, int q, int blk, int t) {
-  const int kind = __ldg(&P.bc[cls].kind);
-  if (kind == LBM_BC_OUTFLOW) return T(0);
-  const int o = (q == 0) ? 0 : ((q & 1) ? q + 1 : q - 1);
-  T v = __ldg(P.src + ((size_t)blk * Q + o) * kCells + t);
-  if (kind == LBM_BC_VELOCITY) {
-    const double eu = c_ex[q] * __ldg(&P.bc[cls].u[0]) + c_ey[q] * __ldg(&P.bc[cls].u[1]) +
-                      c_ez[q] * __ldg(&P.bc[cls].u[2]);
-    v += T(6.0 * wq_rt<Q>(q) * 1.0 * eu);
-  }
-  return v;
-}
+// A fluid leaf's links whose source is not a plain same-level neighbour were
+// resolved by the host builder into records (lattice.h kLink*).  The kernel
+// reads them in batches of four and issues the four source loads back to back:
+//   kLinkSame / kLinkCoarse  -> one load from C_L^k / C_{L-1}^{ceil(k/2)}
+//                               (Explosion, Eq.10);
+//   kLinkBC / kLinkFace      -> halfway bounce-back of the cell's own
+//                               post-collision opposite population, + 6 w_q
+//                               e_q.u_w for a moving wall / inlet, g = 0
+//                               (f = w_q) for outflow;
+//   kLinkCoal                -> (sum_B C_{L+1}^{2k-1} + sum_B C_{L+1}^{2k})/(2|B|)
+//                               (Coalescence, Eq.11, R-A2/R-A3), summed
+//                               in candidate order like the oracle.
+__device__ __forceinline__ int opp_rt(int q) { return q == 0 ? 0 : ((q & 1) ? q + 1 : q - 1); }
 
 template <int Q, typename T>
-__device__ __forceinline__ T slow_link(const StepParams<T>& P, int q, int blk, int t, int px, int py, int pz) {
-  const int exq = c_ex[q], eyq = c_ey[q], ezq = c_ez[q];
-  int s[3] = {px - exq, py - eyq, pz - ezq};
-  int out[3] = {0, 0, 0};
-  bool outside = false;
+__device__ __forceinline__ void resolve_slow(const StepParams<T>& P, T (&g)[Q], uint32_t slow, unsigned j, int blk,
+                                             int t) {
+  const unsigned own = (unsigned)blk * (unsigned)(Q * kCells) + (unsigned)t;
+  while (slow) {
+    int qb[4];
+    uint2 eb[4];
 #pragma unroll
-  for (int a = 0; a < 3; ++a) {
-    const int n = P.own.n[a];
-    if (s[a] < 0 || s[a] >= n) {
-      if (P.periodic[a]) s[a] += (s[a] < 0) ? n : -n;
-      else { out[a] = (s[a] < 0) ? -1 : 1; outside = true; }
-    }
-  }
-  if (outside) return bc_value<Q, T>(P, __ldg(P.face_cls + (out[0] + 1) + 3 * (out[1] + 1) + 9 * (out[2] + 1)), q, blk, t);
-  int tl;
-  int b = lookup(P.own, s[0], s[1], s[2], tl);
-  unsigned ty = type_at(P.own, b, tl);
-  if (ty == kFluid) return __ldg(P.src + ((size_t)b * Q + q) * kCells + tl);  // Eq.(2)
-  if (is_bc(ty)) return bc_value<Q, T>(P, ty, q, blk, t);
-  if (ty == kAbsent) {
-    // Explosion, Eq.(10): the coarser leaf containing s
-    int cl;
-    const int cb = lookup(P.coarse, s[0] >> 1, s[1] >> 1, s[2] >> 1, cl);
-    const unsigned ct = type_at(P.coarse, cb, cl);
-    if (ct == kFluid) return __ldg(P.csrc + ((size_t)cb * Q + q) * kCells + cl);
-    if (is_bc(ct)) return bc_value<Q, T>(P, ct, q, blk, t);
-    return nan_of<T>();
-  }
-  // Coalescence, Eq.(11): fine fluid leaves beta = 2p - e_q + c, c in {0,1}^3
-  int64_t off[8];
-  int nB = 0;
-  unsigned firstbc = 0;
-#pragma unroll
-  for (int c = 0; c < 8; ++c) {
-    int f[3] = {2 * px - exq + (c >> 2), 2 * py - eyq + ((c >> 1) & 1), 2 * pz - ezq + (c & 1)};
-    bool ok = true;
-#pragma unroll
-    for (int a = 0; a < 3; ++a) {
-      const int n = P.fine.n[a];
-      if (f[a] < 0 || f[a] >= n) {
-        if (P.periodic[a]) f[a] += (f[a] < 0) ? n : -n;
-        else ok = false;
+    for (int b = 0; b < 4; ++b) {
+      qb[b] = -1;
+      eb[b] = make_uint2(0u, 0u);
+      if (slow) {
+        qb[b] = __ffs(slow) - 1;
+        slow &= slow - 1;
+        eb[b] = __ldg(P.links + j);
+        ++j;
       }
     }
-    off[c] = -1;
-    if (!ok) continue;
-    int fl;
-    const int fbk = lookup(P.fine, f[0], f[1], f[2], fl);
-    const unsigned ft = type_at(P.fine, fbk, fl);
-    if (ft == kFluid) {
-      off[c] = ((int64_t)fbk * Q + q) * kCells + fl;
-      ++nB;
-    } else if (is_bc(ft) && firstbc == 0) {
-      firstbc = ft;
+    T v[4];
+#pragma unroll
+    for (int b = 0; b < 4; ++b) {
+      v[b] = T(0);
+      if (qb[b] >= 0) {
+        const unsigned tag = eb[b].y >> 28;
+        const T* base = (tag == kLinkCoarse) ? P.csrc : P.src;
+        const unsigned idx = (tag <= kLinkCoarse) ? eb[b].x : own + (unsigned)(opp_rt(qb[b]) * kCells);
+        v[b] = __ldg(base + idx);
+      }
+    }
+#pragma unroll
+    for (int b = 0; b < 4; ++b) {
+      const int q = qb[b];
+      if (q < 0) continue;
+      const unsigned tag = eb[b].y >> 28;
+      T val = v[b];
+      if (tag == kLinkBC || tag == kLinkFace) {
+        const unsigned cls = (tag == kLinkFace) ? (unsigned)__ldg(P.face_cls + eb[b].x) : eb[b].x;
+        const int kind = __ldg(&P.bc[cls].kind);
+        if (kind == LBM_BC_OUTFLOW) {
+          val = T(0);
+        } else if (kind == LBM_BC_VELOCITY) {
+          const double eu = c_ex[q] * __ldg(&P.bc[cls].u[0]) + c_ey[q] * __ldg(&P.bc[cls].u[1]) +
+                            c_ez[q] * __ldg(&P.bc[cls].u[2]);
+          val += T(6.0 * wq_rt<Q>(q) * 1.0 * eu);
+        }
+      } else if (tag == kLinkCoal) {
+        const unsigned n = eb[b].y & 0xfu;
+        const uint32_t* c = P.coal + eb[b].x;
+        T acc = T(0);
+        for (unsigned m = 0; m < n; ++m) acc += __ldg(P.fa + __ldg(c + m));
+        for (unsigned m = 0; m < n; ++m) acc += __ldg(P.fb + __ldg(c + m));
+        val = acc / T(2 * n);
+      }
+#pragma unroll
+      for (int qq = 0; qq < Q; ++qq)
+        if (qq == q) g[qq] = val;
     }
   }
-  if (nB > 0) {
-    T acc = T(0);
-#pragma unroll
-    for (int c = 0; c < 8; ++c)
-      if (off[c] >= 0) acc += __ldg(P.fa + off[c]);
-#pragma unroll
-    for (int c = 0; c < 8; ++c)
-      if (off[c] >= 0) acc += __ldg(P.fb + off[c]);
-    return acc / T(2 * nB);
-  }
-  if (firstbc) return bc_value<Q, T>(P, firstbc, q, blk, t);
-  return nan_of<T>();
 }
 
 // ---------------------------------------------------------------- fused kernel
@@ -352,7 +328,7 @@ __device__ __forceinline__ void process_cell(const StepParams<T>& P, int blk, in
   const int slot = __shfl_sync(FULL, rec, kRecSlot);
   T g[Q];
   if (!STREAM) {
-    if (slot >= 0 && !(__ldg(P.cellinfo + (unsigned)slot * kCells + t) & kFluidBit)) return;
+    if (slot >= 0 && !(__ldg(P.cellinfo + (unsigned)slot * kCells + t).x & kFluidBit)) return;
 #pragma unroll
     for (int q = 0; q < Q; ++q) g[q] = __ldg(P.src + ((unsigned)blk * Q + q) * kCells + t);
     collide<Q, COLL, T>(g, P.omega);
@@ -367,47 +343,67 @@ __device__ __forceinline__ void process_cell(const StepParams<T>& P, int blk, in
     store_cell<Q, T>(g, P.dst, blk, t);
     return;
   }
-  const uint32_t info = __ldg(P.cellinfo + (unsigned)slot * kCells + t);
+  const uint2 ci = __ldg(P.cellinfo + (unsigned)slot * kCells + t);
+  const uint32_t info = ci.x;
   const bool fluid = (info & kFluidBit) != 0;
   const uint32_t need = fluid ? ~info : 0u;
   pull_all<Q, T, true>(g, P.src, G, rec, blk, need, std::make_integer_sequence<int, Q>{});
   if (!fluid) return;
-  uint32_t slow = info & ((1u << Q) - 1u);
-  if (slow) {
-    const int lx = t & 7, ly = (t >> 3) & 7, lz = t >> 6;
-    const int px = __ldg(P.origin + 3 * blk) * kBlock + lx;
-    const int py = __ldg(P.origin + 3 * blk + 1) * kBlock + ly;
-    const int pz = __ldg(P.origin + 3 * blk + 2) * kBlock + lz;
-    while (slow) {
-      const int q = __ffs(slow) - 1;
-      slow &= slow - 1;
-      const T v = slow_link<Q, T>(P, q, blk, t, px, py, pz);
-#pragma unroll
-      for (int qq = 0; qq < Q; ++qq)
-        if (qq == q) g[qq] = v;
-    }
-  }
+  const uint32_t slow = info & ((1u << Q) - 1u);
+  if (slow) resolve_slow<Q, T>(P, g, slow, ci.y, blk, t);
   collide<Q, COLL, T>(g, P.omega);
   store_cell<Q, T>(g, P.dst, blk, t);
 }
 
+// Minimum resident CTAs per SM for the plain-block kernel (register budget:
+// 65536 / (256 * MINB)), chosen per variant from ptxas -v (no spills).
+#ifndef LBMR_OCC_Q19F
+#define LBMR_OCC_Q19F 6
+#endif
 template <int Q, typename T>
-struct Occ { static constexpr int value = 1; };
-template <>
-struct Occ<19, float> { static constexpr int value = 4; };
+struct PlainOcc { static constexpr int value = (Q == 19 && sizeof(T) == 4) ? LBMR_OCC_Q19F : (sizeof(T) == 4 ? 3 : 2); };
 
-// CTA = half an 8^3 block (256 threads, one cell each).
-template <int Q, int COLL, typename T, bool STREAM>
-__global__ void __launch_bounds__(256, Occ<Q, T>::value) level_step_kernel(const StepParams<T> P) {
-  process_cell<Q, COLL, T, STREAM>(P, blockIdx.x >> 1, ((blockIdx.x & 1) << 8) | threadIdx.x);
+// F_L^k over the plain blocks: CTA = half an 8^3 block, one cell per thread.
+template <int Q, int COLL, typename T>
+__global__ void __launch_bounds__(256, PlainOcc<Q, T>::value) level_step_plain(const StepParams<T> P) {
+  const int blk = __ldg(P.ids + (blockIdx.x >> 1));
+  const int t = ((blockIdx.x & 1) << 8) | threadIdx.x;
+  const int rec = __ldg(P.nbr + blk * kRec + (threadIdx.x & 31));
+  const PullGeom G(t);
+  T g[Q];
+  pull_all<Q, T, false>(g, P.src, G, rec, blk, 0u, std::make_integer_sequence<int, Q>{});
+  collide<Q, COLL, T>(g, P.omega);
+  store_cell<Q, T>(g, P.dst, blk, t);
 }
 
-// Persistent variant: gridDim.x = resident CTAs; each CTA walks half-blocks.
-template <int Q, int COLL, typename T, bool STREAM>
-__global__ void __launch_bounds__(256, Occ<Q, T>::value) level_step_persistent(const StepParams<T> P) {
-  const int n = 2 * P.nfluid;
-  for (int w = blockIdx.x; w < n; w += gridDim.x)
-    process_cell<Q, COLL, T, STREAM>(P, w >> 1, ((w & 1) << 8) | threadIdx.x);
+// F_L^k over all fluid blocks in storage (Morton) order; the per-block branch
+// on the record's special slot is warp-uniform.
+template <int Q, int COLL, typename T>
+__global__ void __launch_bounds__(256, PlainOcc<Q, T>::value) level_step_all(const StepParams<T> P) {
+  const int blk = blockIdx.x >> 1;
+  const int t = ((blockIdx.x & 1) << 8) | threadIdx.x;
+  const int rec = __ldg(P.nbr + blk * kRec + (threadIdx.x & 31));
+  if (__shfl_sync(0xffffffffu, rec, kRecSlot) >= 0) {
+    process_cell<Q, COLL, T, true>(P, blk, t);
+    return;
+  }
+  const PullGeom G(t);
+  T g[Q];
+  pull_all<Q, T, false>(g, P.src, G, rec, blk, 0u, std::make_integer_sequence<int, Q>{});
+  collide<Q, COLL, T>(g, P.omega);
+  store_cell<Q, T>(g, P.dst, blk, t);
+}
+
+// F_L^k over the special blocks (interfaces, BCs, domain faces).
+template <int Q, int COLL, typename T>
+__global__ void __launch_bounds__(256) level_step_special(const StepParams<T> P) {
+  process_cell<Q, COLL, T, true>(P, __ldg(P.ids + (blockIdx.x >> 1)), ((blockIdx.x & 1) << 8) | threadIdx.x);
+}
+
+// Prologue C_L^1: collision of the initial state, all fluid blocks.
+template <int Q, int COLL, typename T>
+__global__ void __launch_bounds__(256) level_collide(const StepParams<T> P) {
+  process_cell<Q, COLL, T, false>(P, blockIdx.x >> 1, ((blockIdx.x & 1) << 8) | threadIdx.x);
 }
 
 // ---------------------------------------------------------------- init / macroscopic
@@ -473,31 +469,19 @@ __global__ void __launch_bounds__(512) macroscopic_kernel(const T* pop, const ui
 }
 
 // ---------------------------------------------------------------- dispatch
-static int g_variant = -1;  // 0: one CTA per half block, 1: persistent
-static int g_nsm = 0;
-
 template <int Q, int COLL, typename T>
 static void launch_typed(int kind, const void* params, cudaStream_t s) {
   const StepParams<T>& p = *static_cast<const StepParams<T>*>(params);
-  if (p.nfluid <= 0) return;
-  if (g_variant < 0) {
-    const char* v = getenv("LBMR_VARIANT");
-    g_variant = v ? atoi(v) : 0;
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&g_nsm, cudaDevAttrMultiProcessorCount, dev);
-  }
   dim3 block(256);
-  if (g_variant == 1 && kind == 0) {
-    int occ = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, level_step_persistent<Q, COLL, T, true>, 256, 0);
-    int grid = std::min(2 * p.nfluid, std::max(1, occ) * g_nsm);
-    level_step_persistent<Q, COLL, T, true><<<grid, block, 0, s>>>(p);
-    return;
+  if (kind == 1) {
+    if (p.nfluid > 0) level_collide<Q, COLL, T><<<2 * p.nfluid, block, 0, s>>>(p);
+  } else if (kind == 0) {
+    if (p.nids > 0) level_step_plain<Q, COLL, T><<<2 * p.nids, block, 0, s>>>(p);
+  } else if (kind == 3) {
+    if (p.nfluid > 0) level_step_all<Q, COLL, T><<<2 * p.nfluid, block, 0, s>>>(p);
+  } else {
+    if (p.nids > 0) level_step_special<Q, COLL, T><<<2 * p.nids, block, 0, s>>>(p);
   }
-  dim3 grid(2 * p.nfluid);
-  if (kind == 0) level_step_kernel<Q, COLL, T, true><<<grid, block, 0, s>>>(p);
-  else level_step_kernel<Q, COLL, T, false><<<grid, block, 0, s>>>(p);
 }
 
 void launch_level_step(int Q, int collision, int precision, int kind, const void* params, cudaStream_t s) {

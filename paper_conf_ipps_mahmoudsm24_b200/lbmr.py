@@ -13,7 +13,7 @@ from typing import Optional, Sequence
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "_lib", "liblbmr.so")
+LIB_PATH = os.environ.get("LBMR_LIB") or os.path.join(_HERE, "_lib", "liblbmr.so")
 
 LBM_OK = 0
 STATUS = {0: "LBM_OK", 1: "LBM_E_INVAL", 2: "LBM_E_TILING", 3: "LBM_E_UNBALANCED", 4: "LBM_E_OOM",
