@@ -149,6 +149,28 @@ const char* lbm_last_error(void);
 /* Library version string. */
 const char* lbm_version(void);
 
+/* ---- host-only helpers (no CUDA device needed) -------------------------- */
+
+/* Validate masks and build the block tables on the host only, filling the
+ * counts of `info` (levels, Q, leaves, blocks, special blocks/cells,
+ * kernels_per_step); device_bytes is the population + table footprint the
+ * grid would allocate.  Same validation and error codes as lbm_grid_create. */
+lbm_status lbm_grid_analyze(const lbm_grid_desc* desc, int32_t levels, const uint8_t* const* masks,
+                            lbm_grid_info* info);
+
+/* The pipelined launch order of coarse step n (0-based) for `levels` levels:
+ * writes pairs (level, k) of F_L^k (stream substep k of level L, collide
+ * substep k+1) into order[2*i], order[2*i+1] for i < 2^levels - 1.  Returns
+ * the number of launches, or -1 if levels is out of [1, 16] / order is NULL. */
+int32_t lbm_schedule(int32_t levels, int64_t n, int64_t* order, int32_t capacity);
+
+/* The library's lattice: e[Q][3] velocities and w[Q] weights in the order the
+ * kernels use (rest first, then opposite pairs).  Returns Q, or -1. */
+int32_t lbm_lattice_table(int32_t Q, int32_t* e, double* w);
+
+/* Relaxation rate of level L from omega0, Eq.(9) P:L100. */
+double lbm_omega_level(double omega0, int32_t level);
+
 #ifdef __cplusplus
 }
 #endif

@@ -271,10 +271,33 @@ const char* lbm_last_error(void) { return g_err.c_str(); }
 
 const char* lbm_version(void) { return "lbmr 0.1 (sm_100a)"; }
 
-lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t* const* masks, lbm_grid** out) {
-  g_err.clear();
-  if (!d || !masks || !out) return fail(LBM_E_INVAL, "NULL argument");
-  *out = nullptr;
+int32_t lbm_schedule(int32_t levels, int64_t n, int64_t* order, int32_t capacity) {
+  if (levels < 1 || levels > 16 || !order) return -1;
+  std::vector<std::pair<int, int64_t>> o;
+  step_order(levels, n, o);
+  if ((int64_t)capacity < (int64_t)o.size()) return -1;
+  for (size_t i = 0; i < o.size(); ++i) {
+    order[2 * i] = o[i].first;
+    order[2 * i + 1] = o[i].second;
+  }
+  return (int32_t)o.size();
+}
+
+int32_t lbm_lattice_table(int32_t Q, int32_t* e, double* w) {
+  if ((Q != 19 && Q != 27) || !e || !w) return -1;
+  for (int q = 0; q < Q; ++q) {
+    e[3 * q] = kEx[q];
+    e[3 * q + 1] = kEy[q];
+    e[3 * q + 2] = kEz[q];
+    w[q] = Q == 19 ? weight<19>(q) : weight<27>(q);
+  }
+  return Q;
+}
+
+double lbm_omega_level(double omega0, int32_t level) { return omega_level(omega0, level); }
+
+static lbm_status validate_desc(const lbm_grid_desc* d, int32_t levels, const uint8_t* const* masks) {
+  if (!d || !masks) return fail(LBM_E_INVAL, "NULL argument");
   if (levels < 1 || levels > 16) return fail(LBM_E_INVAL, "levels must be in [1,16]");
   if (d->nx < 1 || d->ny < 1 || d->nz < 1) return fail(LBM_E_INVAL, "nx, ny, nz must be >= 1");
   for (int L = 0; L < levels; ++L)
@@ -297,6 +320,67 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     int64_t n0 = (int64_t)d->nx << L, n1 = (int64_t)d->ny << L, n2 = (int64_t)d->nz << L;
     if (n0 > (1 << 28) || n1 > (1 << 28) || n2 > (1 << 28)) return fail(LBM_E_INVAL, "level too large");
   }
+  return LBM_OK;
+}
+
+static lbm_status build_host(const lbm_grid_desc* d, int32_t levels, const uint8_t* const* masks,
+                             std::vector<HostLevel>& host) {
+  BuildInput in{};
+  in.n0[0] = d->nx; in.n0[1] = d->ny; in.n0[2] = d->nz;
+  for (int a = 0; a < 3; ++a) in.periodic[a] = d->periodic[a] ? 1 : 0;
+  in.levels = levels;
+  in.Q = d->lattice;
+  in.masks = masks;
+  std::string err;
+  int st = build_grid(in, host, err);
+  if (st) return fail((lbm_status)st, err);
+  for (int L = 0; L < levels; ++L)
+    if ((uint64_t)host[L].nblocks * (uint64_t)d->lattice * kCells >= (1ull << 32))
+      return fail(LBM_E_UNSUPPORTED, "level " + std::to_string(L) +
+                                         " too large for one device (> 2^32 populations); use more ranks");
+  return LBM_OK;
+}
+
+static void fill_info(const std::vector<HostLevel>& host, int Q, int prec, lbm_grid_info* info) {
+  std::memset(info, 0, sizeof(*info));
+  info->levels = (int32_t)host.size();
+  info->Q = Q;
+  info->precision = prec;
+  info->kernels_per_step = (1 << host.size()) - 1;
+  for (size_t L = 0; L < host.size(); ++L) {
+    info->leaves[L] = host[L].leaves;
+    info->blocks[L] = host[L].nfluid;
+    info->special_blocks[L] = host[L].nspecial;
+    info->special_cells[L] = host[L].special_cells;
+    info->total_blocks[L] = host[L].nblocks;
+  }
+}
+
+lbm_status lbm_grid_analyze(const lbm_grid_desc* d, int32_t levels, const uint8_t* const* masks,
+                            lbm_grid_info* info) {
+  g_err.clear();
+  if (!info) return fail(LBM_E_INVAL, "NULL info");
+  lbm_status s = validate_desc(d, levels, masks);
+  if (s) return s;
+  std::vector<HostLevel> host;
+  if ((s = build_host(d, levels, masks, host))) return s;
+  fill_info(host, d->lattice, d->precision, info);
+  const int64_t ts = d->precision == LBM_FP32 ? 4 : 8;
+  int64_t bytes = 0;
+  for (const HostLevel& H : host)
+    bytes += 2 * (int64_t)H.nfluid * d->lattice * kCells * ts + (int64_t)H.blkmap.size() * 4 +
+             (int64_t)H.types.size() + (int64_t)H.nbr.size() * 4 + (int64_t)H.cellinfo.size() * 4 +
+             (int64_t)H.links.size() * 4 + (int64_t)H.coal.size() * 4 + (int64_t)H.origin.size() * 4;
+  info->device_bytes = bytes;
+  return LBM_OK;
+}
+
+lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t* const* masks, lbm_grid** out) {
+  g_err.clear();
+  if (!out) return fail(LBM_E_INVAL, "NULL argument");
+  *out = nullptr;
+  lbm_status vs = validate_desc(d, levels, masks);
+  if (vs) return vs;
 
   lbm_grid* g = new lbm_grid();
   g->desc = *d;
@@ -310,27 +394,11 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     g->bc_host[c].pad_ = 0;
     g->bc_host[c].u[0] = g->bc_host[c].u[1] = g->bc_host[c].u[2] = 0.0;
   }
-  BuildInput in{};
-  in.n0[0] = d->nx; in.n0[1] = d->ny; in.n0[2] = d->nz;
-  for (int a = 0; a < 3; ++a) in.periodic[a] = d->periodic[a] ? 1 : 0;
-  in.levels = levels;
-  in.Q = g->Q;
-  in.masks = masks;
-  std::string err;
-  int st = build_grid(in, g->host, err);
-  if (st) {
+  if ((vs = build_host(d, levels, masks, g->host))) {
     delete g;
-    return fail((lbm_status)st, err);
+    return vs;
   }
-  for (int L = 0; L < levels; ++L) {
-    g->omega.push_back(omega_level(d->omega0, L));
-    // kernels index populations with 32-bit offsets
-    if ((uint64_t)g->host[L].nblocks * (uint64_t)g->Q * kCells >= (1ull << 32)) {
-      delete g;
-      return fail(LBM_E_UNSUPPORTED, "level " + std::to_string(L) +
-                                         " too large for one device (> 2^32 populations); use more ranks");
-    }
-  }
+  for (int L = 0; L < levels; ++L) g->omega.push_back(omega_level(d->omega0, L));
 
   auto cleanup = [&](lbm_status s) {
     std::string keep = g_err;
@@ -607,18 +675,7 @@ lbm_status lbm_stats(lbm_grid* g, int64_t* leaves, double* mass) {
 lbm_status lbm_grid_get_info(const lbm_grid* g, lbm_grid_info* info) {
   g_err.clear();
   if (!g || !info) return fail(LBM_E_INVAL, "NULL argument");
-  std::memset(info, 0, sizeof(*info));
-  info->levels = g->levels;
-  info->Q = g->Q;
-  info->precision = g->prec;
-  info->kernels_per_step = (1 << g->levels) - 1;
-  for (int L = 0; L < g->levels; ++L) {
-    info->leaves[L] = g->host[L].leaves;
-    info->blocks[L] = g->host[L].nfluid;
-    info->special_blocks[L] = g->host[L].nspecial;
-    info->special_cells[L] = g->host[L].special_cells;
-    info->total_blocks[L] = g->host[L].nblocks;
-  }
+  fill_info(g->host, g->Q, g->prec, info);
   info->device_bytes = g->device_bytes;
   info->steps_done = g->steps;
   return LBM_OK;

@@ -55,7 +55,8 @@ class GridInfo(ctypes.Structure):
 
 EXPORTS = ["lbm_grid_create", "lbm_set_bc", "lbm_init_equilibrium", "lbm_init_uniform", "lbm_step",
            "lbm_macroscopic", "lbm_stats", "lbm_grid_get_info", "lbm_profile_levels", "lbm_synchronize",
-           "lbm_grid_destroy", "lbm_last_error", "lbm_version"]
+           "lbm_grid_destroy", "lbm_last_error", "lbm_version", "lbm_grid_analyze", "lbm_schedule",
+           "lbm_lattice_table", "lbm_omega_level"]
 
 _lib = None
 
@@ -84,6 +85,14 @@ def load_library(path: str = LIB_PATH):
     lib.lbm_synchronize.argtypes = [P]
     lib.lbm_grid_destroy.argtypes = [P]
     lib.lbm_grid_destroy.restype = None
+    lib.lbm_grid_analyze.argtypes = [ctypes.POINTER(GridDesc), ctypes.c_int32, ctypes.POINTER(ctypes.c_void_p),
+                                     ctypes.POINTER(GridInfo)]
+    lib.lbm_schedule.argtypes = [ctypes.c_int32, ctypes.c_int64, lp, ctypes.c_int32]
+    lib.lbm_schedule.restype = ctypes.c_int32
+    lib.lbm_lattice_table.argtypes = [ctypes.c_int32, ctypes.POINTER(ctypes.c_int32), dp]
+    lib.lbm_lattice_table.restype = ctypes.c_int32
+    lib.lbm_omega_level.argtypes = [ctypes.c_double, ctypes.c_int32]
+    lib.lbm_omega_level.restype = ctypes.c_double
     lib.lbm_last_error.restype = ctypes.c_char_p
     lib.lbm_version.restype = ctypes.c_char_p
     for name in EXPORTS:
@@ -105,6 +114,62 @@ def _dp(a: Optional[np.ndarray]):
     return a.ctypes.data_as(ctypes.POINTER(ctypes.c_double))
 
 
+def make_desc(nx, ny, nz, periodic=(0, 0, 0), face_bc=(0,) * 6, lattice=D3Q19, collision=BGK, precision=FP32,
+              omega0=1.0, stream=None, n_ranks=1, rank=0) -> GridDesc:
+    d = GridDesc()
+    d.nx, d.ny, d.nz = nx, ny, nz
+    for a in range(3):
+        d.periodic[a] = int(periodic[a])
+    for f in range(6):
+        d.face_bc[f] = int(face_bc[f])
+    d.lattice, d.collision, d.precision = int(lattice), int(collision), int(precision)
+    d.omega0 = float(omega0)
+    d.n_ranks, d.rank = int(n_ranks), int(rank)
+    d.stream = stream
+    return d
+
+
+def analyze(nx, ny, nz, masks, **kw) -> GridInfo:
+    """Host-only validation + block tables (no GPU): returns the grid counts."""
+    lib = load_library()
+    ms = [np.ascontiguousarray(m, dtype=np.uint8) for m in masks]
+    d = make_desc(nx, ny, nz, **kw)
+    ptrs = (ctypes.c_void_p * len(ms))(*[m.ctypes.data for m in ms])
+    gi = GridInfo()
+    _check(lib.lbm_grid_analyze(ctypes.byref(d), len(ms), ptrs, ctypes.byref(gi)))
+    return gi
+
+
+def analyze_problem(prob, precision=FP32) -> GridInfo:
+    return analyze(prob.nx, prob.ny, prob.nz, prob.masks, periodic=prob.periodic, face_bc=prob.face_bc,
+                   lattice=prob.Q, collision=KBC if prob.collision == "kbc" else BGK, precision=precision,
+                   omega0=prob.omega0)
+
+
+def schedule(levels: int, n: int = 0):
+    """Pipelined launch order [(L, k), ...] of coarse step n."""
+    lib = load_library()
+    cap = (1 << levels) + 1
+    buf = np.zeros(2 * cap, dtype=np.int64)
+    m = lib.lbm_schedule(int(levels), int(n), buf.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)), cap)
+    if m < 0:
+        raise ValueError("bad levels")
+    return [(int(buf[2 * i]), int(buf[2 * i + 1])) for i in range(m)]
+
+
+def lattice_table(Q: int):
+    lib = load_library()
+    e = np.zeros(3 * Q, dtype=np.int32)
+    w = np.zeros(Q)
+    if lib.lbm_lattice_table(Q, e.ctypes.data_as(ctypes.POINTER(ctypes.c_int32)), _dp(w)) != Q:
+        raise ValueError("bad Q")
+    return e.reshape(Q, 3), w
+
+
+def omega_level(omega0: float, level: int) -> float:
+    return load_library().lbm_omega_level(float(omega0), int(level))
+
+
 class Grid:
     """A multi-level LBM grid on the current CUDA device (one per rank)."""
 
@@ -119,16 +184,7 @@ class Grid:
         for L, m in enumerate(self._masks):
             if m.shape != (nx << L, ny << L, nz << L):
                 raise ValueError(f"mask {L} has shape {m.shape}, expected {(nx << L, ny << L, nz << L)}")
-        d = GridDesc()
-        d.nx, d.ny, d.nz = nx, ny, nz
-        for a in range(3):
-            d.periodic[a] = int(periodic[a])
-        for f in range(6):
-            d.face_bc[f] = int(face_bc[f])
-        d.lattice, d.collision, d.precision = int(lattice), int(collision), int(precision)
-        d.omega0 = float(omega0)
-        d.n_ranks, d.rank = 1, 0
-        d.stream = stream
+        d = make_desc(nx, ny, nz, periodic, face_bc, lattice, collision, precision, omega0, stream)
         ptrs = (ctypes.c_void_p * self.levels)(*[m.ctypes.data for m in self._masks])
         h = ctypes.c_void_p()
         _check(lib.lbm_grid_create(ctypes.byref(d), self.levels, ptrs, ctypes.byref(h)))
