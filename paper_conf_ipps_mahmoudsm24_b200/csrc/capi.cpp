@@ -77,8 +77,6 @@ struct lbm_grid {
   uint8_t* face_dev = nullptr;
   cudaStream_t stream = nullptr;
   bool own_stream = false;
-  cudaStream_t side = nullptr;          // special blocks run beside the plain ones
-  cudaEvent_t fork = nullptr, join = nullptr;
   cudaGraphExec_t graph[2] = {nullptr, nullptr};
   bool needs_prologue = true;
   bool init_locked = false;  // a step ran since the last init_uniform
@@ -186,26 +184,7 @@ void launch_F_typed(lbm_grid* g, int L, int64_t k, int kind) {
     launch_level_step(g->Q, g->coll, g->prec, 1, &p, g->stream);
     return;
   }
-  const HostLevel& H = g->host[L];
-  static int split = -1;
-  if (split < 0) split = getenv("LBMR_SPLIT") ? atoi(getenv("LBMR_SPLIT")) : 0;
-  if (!split) {  // one launch over all blocks in Morton order
-    launch_level_step(g->Q, g->coll, g->prec, 3, &p, g->stream);
-    return;
-  }
-  // fork: special blocks on the side stream, plain blocks on the main stream
-  if (H.special_ids.size()) {
-    cudaEventRecord(g->fork, g->stream);
-    cudaStreamWaitEvent(g->side, g->fork, 0);
-    p.ids = g->dev[L].special_ids;
-    p.nids = (int32_t)H.special_ids.size();
-    launch_level_step(g->Q, g->coll, g->prec, 2, &p, g->side);
-    cudaEventRecord(g->join, g->side);
-  }
-  p.ids = g->dev[L].plain_ids;
-  p.nids = (int32_t)H.plain_ids.size();
   launch_level_step(g->Q, g->coll, g->prec, 0, &p, g->stream);
-  if (H.special_ids.size()) cudaStreamWaitEvent(g->stream, g->join, 0);
 }
 
 void launch_F(lbm_grid* g, int L, int64_t k, int kind) {
@@ -415,10 +394,7 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     }
     g->own_stream = true;
   }
-  if (cudaStreamCreateWithFlags(&g->side, cudaStreamNonBlocking) != cudaSuccess ||
-      cudaEventCreateWithFlags(&g->fork, cudaEventDisableTiming) != cudaSuccess ||
-      cudaEventCreateWithFlags(&g->join, cudaEventDisableTiming) != cudaSuccess)
-    return cleanup(fail(LBM_E_CUDA, "stream/event creation failed"));
+
   g->dev.resize(levels);
   lbm_status s;
   for (int L = 0; L < levels; ++L) {
@@ -686,11 +662,7 @@ void lbm_grid_destroy(lbm_grid* g) {
   if (g->stream) cudaStreamSynchronize(g->stream);
   for (int p = 0; p < 2; ++p)
     if (g->graph[p]) cudaGraphExecDestroy(g->graph[p]);
-  if (g->side) cudaStreamSynchronize(g->side);
   for (void* p : g->allocs) cudaFree(p);
-  if (g->fork) cudaEventDestroy(g->fork);
-  if (g->join) cudaEventDestroy(g->join);
-  if (g->side) cudaStreamDestroy(g->side);
   if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
   delete g;
 }

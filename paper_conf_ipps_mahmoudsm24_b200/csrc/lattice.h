@@ -40,12 +40,16 @@ LBM_HD constexpr int nbr_slot(int dx, int dy, int dz) { return (dx + 1) + 3 * (d
 constexpr int kBlock = 8;            // B = 8 (B compile time)
 constexpr int kCells = 512;          // B^3
 constexpr unsigned kFluidBit = 1u << 31;
-// per-fluid-block record of 32 int32 (one 128-byte line, loaded by one warp
-// instruction): [0..26] neighbour block ids by nbr_slot (-1 none), [27]
-// special slot (-1 plain), [28..30] block coordinates, [31] unused
-constexpr int kRec = 32;
+// per-fluid-block record of 64 int32 (two 128-byte lines, one warp load
+// each): [0..26] neighbour block ids by nbr_slot (-1: none, outside, or a
+// block without fluid leaves), [27] special slot (-1 plain), [28..30] block
+// coordinates, [31] unused, [32+w] fluid-leaf mask of warp w (cells 32w..32w+31),
+// [48+w] mask of the fluid leaves of warp w that have a slow link
+constexpr int kRec = 64;
 constexpr int kRecSlot = 27;
 constexpr int kRecOrigin = 28;
+constexpr int kRecFluid = 32;
+constexpr int kRecSpecial = 48;
 
 // slow-link record {w0, w1}: tag = w1 >> 28
 //  kLinkSame   w0 = population index at level L (irregular same-level source)

@@ -292,21 +292,25 @@ struct PullGeom {
   }
 };
 
+// PRED = false: every link is a plain same-level pull.  PRED = true: load
+// only for fluid cells and existing neighbour blocks (links flagged slow are
+// loaded speculatively from the block arithmetic's source and overwritten by
+// resolve_slow; the source memory always exists).
 template <int Q, typename T, bool PRED, int q>
 __device__ __forceinline__ void pull_one(T (&g)[Q], const T* __restrict__ src, const PullGeom& G, int rec, int blk,
-                                         uint32_t need) {
+                                         bool fluid) {
   constexpr unsigned FULL = 0xffffffffu;
   const int nb = (q == 0) ? blk : __shfl_sync(FULL, rec, G.slot<q>());
   const unsigned off = (unsigned)nb * (unsigned)(Q * kCells) + (unsigned)G.local<q>();
   const T* p = src + q * kCells;  // constant part folds into the load's immediate offset
-  if (PRED) g[q] = (need & (1u << q)) ? __ldg(p + off) : T(0);
+  if (PRED) g[q] = (fluid && nb >= 0) ? __ldg(p + off) : T(0);
   else g[q] = __ldg(p + off);
 }
 
 template <int Q, typename T, bool PRED, int... qs>
 __device__ __forceinline__ void pull_all(T (&g)[Q], const T* __restrict__ src, const PullGeom& G, int rec, int blk,
-                                         uint32_t need, std::integer_sequence<int, qs...>) {
-  (pull_one<Q, T, PRED, qs>(g, src, G, rec, blk, need), ...);
+                                         bool fluid, std::integer_sequence<int, qs...>) {
+  (pull_one<Q, T, PRED, qs>(g, src, G, rec, blk, fluid), ...);
 }
 
 template <int Q, typename T>
@@ -316,94 +320,65 @@ __device__ __forceinline__ void store_cell(const T (&g)[Q], T* __restrict__ dst,
   for (int q = 0; q < Q; ++q) d[q * kCells] = g[q];
 }
 
-// One cell (blk, t) of F_L^k.  No shared memory and no barrier: each warp
-// loads its block's 128-byte record (27 neighbour ids, special slot, origin)
-// with one coalesced load and picks neighbour ids with __shfl_sync.  Blocks
-// without special cells (the bulk) take a branch-free pull; the branch on the
-// block's slot is warp-uniform.  Offsets are 32-bit (host-checked).
-template <int Q, int COLL, typename T, bool STREAM>
-__device__ __forceinline__ void process_cell(const StepParams<T>& P, int blk, int t) {
-  constexpr unsigned FULL = 0xffffffffu;
-  const int rec = __ldg(P.nbr + blk * kRec + (threadIdx.x & 31));
-  const int slot = __shfl_sync(FULL, rec, kRecSlot);
-  T g[Q];
-  if (!STREAM) {
-    if (slot >= 0 && !(__ldg(P.cellinfo + (unsigned)slot * kCells + t).x & kFluidBit)) return;
-#pragma unroll
-    for (int q = 0; q < Q; ++q) g[q] = __ldg(P.src + ((unsigned)blk * Q + q) * kCells + t);
-    collide<Q, COLL, T>(g, P.omega);
-    store_cell<Q, T>(g, P.dst, blk, t);
-    return;
-  }
-  const PullGeom G(t);
-  if (slot < 0) {
-    // plain block: every cell is a fluid leaf with only same-level links
-    pull_all<Q, T, false>(g, P.src, G, rec, blk, 0u, std::make_integer_sequence<int, Q>{});
-    collide<Q, COLL, T>(g, P.omega);
-    store_cell<Q, T>(g, P.dst, blk, t);
-    return;
-  }
-  const uint2 ci = __ldg(P.cellinfo + (unsigned)slot * kCells + t);
-  const uint32_t info = ci.x;
-  const bool fluid = (info & kFluidBit) != 0;
-  const uint32_t need = fluid ? ~info : 0u;
-  pull_all<Q, T, true>(g, P.src, G, rec, blk, need, std::make_integer_sequence<int, Q>{});
-  if (!fluid) return;
-  const uint32_t slow = info & ((1u << Q) - 1u);
-  if (slow) resolve_slow<Q, T>(P, g, slow, ci.y, blk, t);
-  collide<Q, COLL, T>(g, P.omega);
-  store_cell<Q, T>(g, P.dst, blk, t);
-}
-
-// Minimum resident CTAs per SM for the plain-block kernel (register budget:
-// 65536 / (256 * MINB)), chosen per variant from ptxas -v (no spills).
+// Minimum resident CTAs per SM (register budget 65536 / (256 * MINB)),
+// chosen per variant from ptxas -v and measurement.
 #ifndef LBMR_OCC_Q19F
 #define LBMR_OCC_Q19F 6
 #endif
 template <int Q, typename T>
 struct PlainOcc { static constexpr int value = (Q == 19 && sizeof(T) == 4) ? LBMR_OCC_Q19F : (sizeof(T) == 4 ? 3 : 2); };
 
-// F_L^k over the plain blocks: CTA = half an 8^3 block, one cell per thread.
-template <int Q, int COLL, typename T>
-__global__ void __launch_bounds__(256, PlainOcc<Q, T>::value) level_step_plain(const StepParams<T> P) {
-  const int blk = __ldg(P.ids + (blockIdx.x >> 1));
-  const int t = ((blockIdx.x & 1) << 8) | threadIdx.x;
-  const int rec = __ldg(P.nbr + blk * kRec + (threadIdx.x & 31));
-  const PullGeom G(t);
-  T g[Q];
-  pull_all<Q, T, false>(g, P.src, G, rec, blk, 0u, std::make_integer_sequence<int, Q>{});
-  collide<Q, COLL, T>(g, P.omega);
-  store_cell<Q, T>(g, P.dst, blk, t);
-}
-
-// F_L^k over all fluid blocks in storage (Morton) order; the per-block branch
-// on the record's special slot is warp-uniform.
+// F_L^k over all fluid blocks in storage (Morton) order; CTA = half an 8^3
+// block, one cell per thread.  No shared memory and no barrier: each warp
+// reads its block's record (27 neighbour ids, special slot, origin, per-warp
+// fluid and slow-link masks) with one coalesced and two broadcast loads and
+// picks neighbour ids with __shfl_sync.  A warp whose 32 cells are fluid
+// leaves with only same-level links (the bulk) takes the predicate-free pull;
+// the test is warp-uniform.  Other warps load the same way for their fluid
+// cells, and the few cells with slow links then apply their link records.
+// Offsets are 32-bit (host-checked: nblocks * Q * 512 < 2^32).
 template <int Q, int COLL, typename T>
 __global__ void __launch_bounds__(256, PlainOcc<Q, T>::value) level_step_all(const StepParams<T> P) {
+  constexpr unsigned FULL = 0xffffffffu;
   const int blk = blockIdx.x >> 1;
   const int t = ((blockIdx.x & 1) << 8) | threadIdx.x;
-  const int rec = __ldg(P.nbr + blk * kRec + (threadIdx.x & 31));
-  if (__shfl_sync(0xffffffffu, rec, kRecSlot) >= 0) {
-    process_cell<Q, COLL, T, true>(P, blk, t);
-    return;
-  }
+  const int lane = threadIdx.x & 31;
+  const int* R = P.nbr + blk * kRec;
+  const int rec = __ldg(R + lane);
+  const uint32_t fm = (uint32_t)__ldg(R + kRecFluid + (t >> 5));
+  const uint32_t sm = (uint32_t)__ldg(R + kRecSpecial + (t >> 5));
   const PullGeom G(t);
   T g[Q];
-  pull_all<Q, T, false>(g, P.src, G, rec, blk, 0u, std::make_integer_sequence<int, Q>{});
+  if (fm == FULL && sm == 0u) {
+    pull_all<Q, T, false>(g, P.src, G, rec, blk, true, std::make_integer_sequence<int, Q>{});
+    collide<Q, COLL, T>(g, P.omega);
+    store_cell<Q, T>(g, P.dst, blk, t);
+    return;
+  }
+  const int slot = __shfl_sync(FULL, rec, kRecSlot);
+  const bool fluid = (fm >> lane) & 1u;
+  const bool special = (sm >> lane) & 1u;
+  uint2 ci = make_uint2(0u, 0u);
+  if (special) ci = __ldg(P.cellinfo + (unsigned)slot * kCells + t);
+  pull_all<Q, T, true>(g, P.src, G, rec, blk, fluid, std::make_integer_sequence<int, Q>{});
+  if (!fluid) return;
+  if (special) resolve_slow<Q, T>(P, g, ci.x & ((1u << Q) - 1u), ci.y, blk, t);
   collide<Q, COLL, T>(g, P.omega);
   store_cell<Q, T>(g, P.dst, blk, t);
-}
-
-// F_L^k over the special blocks (interfaces, BCs, domain faces).
-template <int Q, int COLL, typename T>
-__global__ void __launch_bounds__(256) level_step_special(const StepParams<T> P) {
-  process_cell<Q, COLL, T, true>(P, __ldg(P.ids + (blockIdx.x >> 1)), ((blockIdx.x & 1) << 8) | threadIdx.x);
 }
 
 // Prologue C_L^1: collision of the initial state, all fluid blocks.
 template <int Q, int COLL, typename T>
 __global__ void __launch_bounds__(256) level_collide(const StepParams<T> P) {
-  process_cell<Q, COLL, T, false>(P, blockIdx.x >> 1, ((blockIdx.x & 1) << 8) | threadIdx.x);
+  const int blk = blockIdx.x >> 1;
+  const int t = ((blockIdx.x & 1) << 8) | threadIdx.x;
+  const uint32_t fm = (uint32_t)__ldg(P.nbr + blk * kRec + kRecFluid + (t >> 5));
+  if (!((fm >> (threadIdx.x & 31)) & 1u)) return;
+  T g[Q];
+#pragma unroll
+  for (int q = 0; q < Q; ++q) g[q] = __ldg(P.src + ((unsigned)blk * Q + q) * kCells + t);
+  collide<Q, COLL, T>(g, P.omega);
+  store_cell<Q, T>(g, P.dst, blk, t);
 }
 
 // ---------------------------------------------------------------- init / macroscopic
@@ -472,16 +447,10 @@ __global__ void __launch_bounds__(512) macroscopic_kernel(const T* pop, const ui
 template <int Q, int COLL, typename T>
 static void launch_typed(int kind, const void* params, cudaStream_t s) {
   const StepParams<T>& p = *static_cast<const StepParams<T>*>(params);
-  dim3 block(256);
-  if (kind == 1) {
-    if (p.nfluid > 0) level_collide<Q, COLL, T><<<2 * p.nfluid, block, 0, s>>>(p);
-  } else if (kind == 0) {
-    if (p.nids > 0) level_step_plain<Q, COLL, T><<<2 * p.nids, block, 0, s>>>(p);
-  } else if (kind == 3) {
-    if (p.nfluid > 0) level_step_all<Q, COLL, T><<<2 * p.nfluid, block, 0, s>>>(p);
-  } else {
-    if (p.nids > 0) level_step_special<Q, COLL, T><<<2 * p.nids, block, 0, s>>>(p);
-  }
+  if (p.nfluid <= 0) return;
+  dim3 block(256), grid(2 * p.nfluid);
+  if (kind == 1) level_collide<Q, COLL, T><<<grid, block, 0, s>>>(p);
+  else level_step_all<Q, COLL, T><<<grid, block, 0, s>>>(p);
 }
 
 void launch_level_step(int Q, int collision, int precision, int kind, const void* params, cudaStream_t s) {
