@@ -171,6 +171,48 @@ int32_t lbm_lattice_table(int32_t Q, int32_t* e, double* w);
 /* Relaxation rate of level L from omega0, Eq.(9) P:L100. */
 double lbm_omega_level(double omega0, int32_t level);
 
+/* ---- x-slab partition (multi-GPU), DESIGN.md §9 ---------------------------
+ * A grid created with desc->n_ranks = P > 1 holds rank desc->rank's slab of
+ * level-0 x cells [cuts[rank], cuts[rank+1]) (cuts from lbm_partition_cuts,
+ * identical on every rank since they depend only on the masks) plus one
+ * level-0 cell of halo on each side that has a neighbour (x periodic: a ring).
+ * Every rank passes the SAME global masks.  Dense arrays of
+ * lbm_init_equilibrium / lbm_macroscopic then cover the owned slab only:
+ * shape ((cuts[rank+1]-cuts[rank])<<L, ny<<L, nz<<L).  Before the first
+ * lbm_step every side with a neighbour must be connected (lbm_halo_connect
+ * with the neighbour's lbm_halo_export blob, or lbm_halo_connect_local for a
+ * grid of the same process); all ranks must then issue the same sequence of
+ * lbm_step / lbm_profile_levels calls.  Side 0 = -x, side 1 = +x. */
+
+/* Balanced cuts (n_ranks + 1 entries) at level-0 cell boundaries: the work of
+ * column x is sum_L 2^L (fluid leaves of level L inside it).  Host only. */
+lbm_status lbm_partition_cuts(const lbm_grid_desc* desc, int32_t levels, const uint8_t* const* masks,
+                              int32_t n_ranks, int32_t* cuts);
+
+/* Owned level-0 x range [x_begin, x_end) of the grid (global coordinates). */
+lbm_status lbm_grid_slab(const lbm_grid* g, int32_t* x_begin, int32_t* x_end);
+
+/* Serialise what the neighbour on `side` needs to write into this grid: the
+ * halo cell lists per level and CUDA IPC handles of the population buffers
+ * and the protocol flags.  blob = NULL returns the size only. */
+lbm_status lbm_halo_export(const lbm_grid* g, int32_t side, void* blob, int64_t capacity, int64_t* size);
+
+/* Connect `side` to the neighbour whose lbm_halo_export(other side) blob is
+ * given (another process; the buffers are opened with CUDA IPC). */
+lbm_status lbm_halo_connect(lbm_grid* g, int32_t side, const void* blob, int64_t size);
+
+/* Connect `side` to a neighbour grid of this process (same device or a
+ * peer-accessible one). */
+lbm_status lbm_halo_connect_local(lbm_grid* g, int32_t side, lbm_grid* peer);
+
+/* Host-only plan of one side/level of rank desc->rank: global coordinates
+ * (x, y, z) of the cells it sends (its first owned layer at the cut) and of
+ * its halo cells (received), in the order both sides use.  xyz arrays hold
+ * 3 * capacity int64 each (may be NULL to query the counts). */
+lbm_status lbm_halo_plan(const lbm_grid_desc* desc, int32_t levels, const uint8_t* const* masks, int32_t side,
+                         int32_t level, int64_t* send_xyz, int64_t* halo_xyz, int64_t capacity, int64_t* n_send,
+                         int64_t* n_halo);
+
 #ifdef __cplusplus
 }
 #endif

@@ -15,6 +15,8 @@
 // alternate) and replayed with cudaGraphLaunch.
 #include <cuda_runtime.h>
 
+#include <unistd.h>
+
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
@@ -54,9 +56,12 @@ struct DevLevel {
   uint32_t* cellinfo = nullptr;
   uint32_t* links = nullptr;
   uint32_t* coal = nullptr;
-  int32_t* plain_ids = nullptr;
-  int32_t* special_ids = nullptr;
+  int32_t* bpeer = nullptr;
   void* pop[2] = {nullptr, nullptr};
+  // neighbour rank on each side: its population buffers and the halo cell
+  // index (in its grid) of every entry of our send list
+  void* peer_pop[2][2] = {{nullptr, nullptr}, {nullptr, nullptr}};
+  uint32_t* peer_cells[2] = {nullptr, nullptr};
 };
 
 }  // namespace
@@ -84,6 +89,15 @@ struct lbm_grid {
   int64_t steps = 0;
   int64_t device_bytes = 0;
   std::vector<void*> allocs;
+  // x-slab partition
+  int n_ranks = 1, rank = 0;
+  std::vector<int32_t> cuts;          // level-0 x cuts, n_ranks + 1 entries
+  int32_t x_lo = 0;                   // global level-0 x of local x = 0
+  int32_t has_nb[2] = {0, 0};
+  bool connected[2] = {false, false};
+  unsigned long long* flags = nullptr;      // [4], see kernels.h
+  unsigned long long* peer_flags[2] = {nullptr, nullptr};
+  std::vector<std::pair<std::string, void*>> ipc_open;  // opened IPC handles
 };
 
 namespace {
@@ -173,7 +187,21 @@ StepParams<T> make_params(const lbm_grid* g, int L, int64_t k) {
   p.omega = (T)g->omega[L];
   for (int a = 0; a < 3; ++a) p.periodic[a] = g->desc.periodic[a];
   p.face_cls = g->face_dev;
-  p.nfluid = g->host[L].nfluid;
+  p.nfluid = g->n_ranks > 1 ? g->host[L].nlaunch : g->host[L].nfluid;
+  if (g->n_ranks > 1) {
+    const HostLevel& H = g->host[L];
+    p.nbctas = std::max(2 * H.nboundary, 1);
+    p.nboundary = H.nboundary;
+    p.flags = g->flags;
+    p.bpeer = D.bpeer;
+    for (int sd = 0; sd < 2; ++sd) {
+      p.has_nb[sd] = g->has_nb[sd];
+      if (!g->has_nb[sd]) continue;
+      p.peer_flag[sd] = g->peer_flags[sd] + (1 - sd);  // we are the peer's neighbour on its other side
+      p.peer_dst[sd] = static_cast<T*>(D.peer_pop[sd][(k + 1) & 1]);
+      p.peer_cells[sd] = D.peer_cells[sd];
+    }
+  }
   return p;
 }
 
@@ -294,7 +322,8 @@ static lbm_status validate_desc(const lbm_grid_desc* d, int32_t levels, const ui
       if (c < 2 || c > 254) return fail(LBM_E_INVAL, "face_bc of a non-periodic face must be a BC class in 2..254");
     }
   }
-  if (d->n_ranks > 1) return fail(LBM_E_UNSUPPORTED, "multi-rank slab partition not enabled in this build");
+  if (d->n_ranks < 1 || d->rank < 0 || d->rank >= d->n_ranks) return fail(LBM_E_INVAL, "bad n_ranks / rank");
+  if (d->n_ranks > d->nx) return fail(LBM_E_INVAL, "more ranks than level-0 x cells");
   for (int L = 0; L < levels; ++L) {
     int64_t n0 = (int64_t)d->nx << L, n1 = (int64_t)d->ny << L, n2 = (int64_t)d->nz << L;
     if (n0 > (1 << 28) || n1 > (1 << 28) || n2 > (1 << 28)) return fail(LBM_E_INVAL, "level too large");
@@ -302,14 +331,90 @@ static lbm_status validate_desc(const lbm_grid_desc* d, int32_t levels, const ui
   return LBM_OK;
 }
 
+// Balanced x-slab cuts at coarse-cell boundaries: the work of
+// level-0 column x is sum_L 2^L * (fluid leaves of level L inside it).
+static void partition_cuts(const lbm_grid_desc* d, int32_t levels, const uint8_t* const* masks, int P,
+                           std::vector<int32_t>& cuts) {
+  const int nx = d->nx;
+  std::vector<double> W(nx, 0.0);
+  for (int L = 0; L < levels; ++L) {
+    const int64_t plane = ((int64_t)d->ny << L) * ((int64_t)d->nz << L);
+    const int64_t nxl = (int64_t)nx << L;
+    std::vector<int64_t> cnt(nxl, 0);
+#pragma omp parallel for schedule(static)
+    for (int64_t x = 0; x < nxl; ++x) {
+      const uint8_t* m = masks[L] + x * plane;
+      int64_t c = 0;
+      for (int64_t i = 0; i < plane; ++i) c += (m[i] == 1);
+      cnt[x] = c;
+    }
+    for (int64_t x = 0; x < nxl; ++x) W[x >> L] += (double)(cnt[x] << L);
+  }
+  std::vector<double> pre(nx + 1, 0.0);
+  for (int x = 0; x < nx; ++x) pre[x + 1] = pre[x] + W[x];
+  cuts.assign(P + 1, 0);
+  cuts[P] = nx;
+  for (int r = 1; r < P; ++r) {
+    const double target = pre[nx] * r / P;
+    int x = (int)(std::lower_bound(pre.begin(), pre.end(), target) - pre.begin());
+    if (x > 0 && target - pre[x - 1] < pre[x] - target) --x;
+    x = std::max(x, cuts[r - 1] + 1);
+    x = std::min(x, nx - (P - r));
+    cuts[r] = x;
+  }
+}
+
+struct LocalSlab {
+  lbm_grid_desc desc;                      // local dims, x non-periodic
+  std::vector<std::vector<uint8_t>> masks; // local masks (slab + halo)
+  std::vector<const uint8_t*> ptrs;
+  int32_t x_lo = 0, owned_lo0 = 0, owned_hi0 = -1, has_nb[2] = {0, 0};
+};
+
+static void make_local(const lbm_grid_desc* d, int32_t levels, const uint8_t* const* masks,
+                       const std::vector<int32_t>& cuts, LocalSlab& out) {
+  const int P = d->n_ranks, r = d->rank;
+  const bool per = d->periodic[0] != 0;
+  out.has_nb[0] = (r > 0 || per) ? 1 : 0;
+  out.has_nb[1] = (r < P - 1 || per) ? 1 : 0;
+  out.x_lo = cuts[r] - out.has_nb[0];
+  const int x_hi = cuts[r + 1] + out.has_nb[1];
+  const int nxl = x_hi - out.x_lo;
+  out.desc = *d;
+  out.desc.nx = nxl;
+  out.desc.periodic[0] = 0;
+  out.owned_lo0 = out.has_nb[0];
+  out.owned_hi0 = nxl - out.has_nb[1];
+  out.masks.resize(levels);
+  for (int L = 0; L < levels; ++L) {
+    const int64_t plane = ((int64_t)d->ny << L) * ((int64_t)d->nz << L);
+    const int64_t gn = (int64_t)d->nx << L, ln = (int64_t)nxl << L;
+    out.masks[L].resize(ln * plane);
+    for (int64_t x = 0; x < ln; ++x) {
+      const int64_t gx = (((int64_t)out.x_lo << L) + x + gn) % gn;
+      std::memcpy(&out.masks[L][x * plane], masks[L] + gx * plane, plane);
+    }
+    out.ptrs.push_back(out.masks[L].data());
+  }
+}
+
 static lbm_status build_host(const lbm_grid_desc* d, int32_t levels, const uint8_t* const* masks,
-                             std::vector<HostLevel>& host) {
+                             std::vector<HostLevel>& host, LocalSlab* slab = nullptr) {
   BuildInput in{};
   in.n0[0] = d->nx; in.n0[1] = d->ny; in.n0[2] = d->nz;
   for (int a = 0; a < 3; ++a) in.periodic[a] = d->periodic[a] ? 1 : 0;
   in.levels = levels;
   in.Q = d->lattice;
   in.masks = masks;
+  if (slab) {
+    in.n0[0] = slab->desc.nx;
+    in.periodic[0] = 0;
+    in.masks = slab->ptrs.data();
+    in.owned_lo0 = slab->owned_lo0;
+    in.owned_hi0 = slab->owned_hi0;
+    in.has_nb[0] = slab->has_nb[0];
+    in.has_nb[1] = slab->has_nb[1];
+  }
   std::string err;
   int st = build_grid(in, host, err);
   if (st) return fail((lbm_status)st, err);
@@ -342,7 +447,15 @@ lbm_status lbm_grid_analyze(const lbm_grid_desc* d, int32_t levels, const uint8_
   lbm_status s = validate_desc(d, levels, masks);
   if (s) return s;
   std::vector<HostLevel> host;
-  if ((s = build_host(d, levels, masks, host))) return s;
+  if (d->n_ranks > 1) {
+    std::vector<int32_t> cuts;
+    partition_cuts(d, levels, masks, d->n_ranks, cuts);
+    LocalSlab slab;
+    make_local(d, levels, masks, cuts, slab);
+    if ((s = build_host(d, levels, masks, host, &slab))) return s;
+  } else if ((s = build_host(d, levels, masks, host))) {
+    return s;
+  }
   fill_info(host, d->lattice, d->precision, info);
   const int64_t ts = d->precision == LBM_FP32 ? 4 : 8;
   int64_t bytes = 0;
@@ -373,7 +486,21 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     g->bc_host[c].pad_ = 0;
     g->bc_host[c].u[0] = g->bc_host[c].u[1] = g->bc_host[c].u[2] = 0.0;
   }
-  if ((vs = build_host(d, levels, masks, g->host))) {
+  g->n_ranks = d->n_ranks;
+  g->rank = d->rank;
+  if (d->n_ranks > 1) {
+    partition_cuts(d, levels, masks, d->n_ranks, g->cuts);
+    LocalSlab slab;
+    make_local(d, levels, masks, g->cuts, slab);
+    g->x_lo = slab.x_lo;
+    g->has_nb[0] = slab.has_nb[0];
+    g->has_nb[1] = slab.has_nb[1];
+    vs = build_host(d, levels, masks, g->host, &slab);
+  } else {
+    g->cuts = {0, d->nx};
+    vs = build_host(d, levels, masks, g->host);
+  }
+  if (vs) {
     delete g;
     return vs;
   }
@@ -395,6 +522,11 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     g->own_stream = true;
   }
 
+  static bool preloaded = false;
+  if (!preloaded) {
+    preload_kernels();
+    preloaded = true;
+  }
   g->dev.resize(levels);
   lbm_status s;
   for (int L = 0; L < levels; ++L) {
@@ -408,8 +540,7 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     if ((s = dev_upload(g, &D.cellinfo, H.cellinfo))) return cleanup(s);
     if ((s = dev_upload(g, &D.links, H.links))) return cleanup(s);
     if ((s = dev_upload(g, &D.coal, H.coal))) return cleanup(s);
-    if ((s = dev_upload(g, &D.plain_ids, H.plain_ids))) return cleanup(s);
-    if ((s = dev_upload(g, &D.special_ids, H.special_ids))) return cleanup(s);
+    if ((s = dev_upload(g, &D.bpeer, H.bpeer))) return cleanup(s);
     for (int b = 0; b < 2; ++b) {
       if ((s = dev_alloc(g, &D.pop[b], pop_bytes(g, L)))) return cleanup(s);
       if (cudaMemset(D.pop[b], 0, pop_bytes(g, L)) != cudaSuccess) return cleanup(fail(LBM_E_CUDA, "memset"));
@@ -422,6 +553,11 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     std::vector<int32_t>().swap(H.nbr);
   }
   void* p;
+  if (g->n_ranks > 1) {  // halo-protocol flags, own allocation so it can be shared by CUDA IPC
+    if ((s = dev_alloc(g, &p, 4 * sizeof(unsigned long long)))) return cleanup(s);
+    if (cudaMemset(p, 0, 4 * sizeof(unsigned long long)) != cudaSuccess) return cleanup(fail(LBM_E_CUDA, "memset"));
+    g->flags = static_cast<unsigned long long*>(p);
+  }
   if ((s = dev_alloc(g, &p, sizeof(BCEntry) * 256))) return cleanup(s);
   g->bc_dev = static_cast<BCEntry*>(p);
   if ((s = dev_alloc(g, &p, 32))) return cleanup(s);
@@ -464,7 +600,8 @@ static lbm_status init_level(lbm_grid* g, int L, const double* rho, const double
       for (int l = 0; l < kCells; ++l) {
         if (H.types[(size_t)b * kCells + l] != kFluid) continue;
         const int64_t x = ox + (l & 7), y = oy + ((l >> 3) & 7), z = oz + (l >> 6);
-        const int64_t c = (x * H.n[1] + y) * H.n[2] + z;
+        if (x < H.owned_lo || x >= H.owned_hi) continue;  // halo cells come from the neighbour
+        const int64_t c = ((x - H.owned_lo) * H.n[1] + y) * H.n[2] + z;
         const size_t k = (size_t)b * kCells + l;
         if (rho) r[k] = rho[c];
         if (u) { v[3 * k] = u[3 * c]; v[3 * k + 1] = u[3 * c + 1]; v[3 * k + 2] = u[3 * c + 2]; }
@@ -518,8 +655,22 @@ lbm_status lbm_step(lbm_grid* g, int32_t n) {
   if (g->broken) return fail(LBM_E_STATE, "grid is in an error state");
   if (n < 0) return fail(LBM_E_INVAL, "n_coarse must be >= 0");
   if (n == 0) return LBM_OK;
+  for (int sd = 0; sd < 2; ++sd)
+    if (g->n_ranks > 1 && g->has_nb[sd] && !g->connected[sd])
+      return fail(LBM_E_STATE, "halo side " + std::to_string(sd) + " not connected");
   lbm_status s;
   if (g->needs_prologue && (s = run_prologue(g))) { g->broken = true; return s; }
+  if (getenv("LBMR_DEBUG_PROLOGUE_ONLY")) return LBM_OK;
+  if (getenv("LBMR_DEBUG_NO_GRAPH")) {
+    std::vector<std::pair<int, int64_t>> order;
+    for (int i = 0; i < n; ++i) {
+      step_order(g->levels, g->steps, order);
+      for (auto& lk : order) launch_F(g, lk.first, lk.second, 0);
+      ++g->steps;
+    }
+    g->init_locked = true;
+    return LBM_OK;
+  }
   if ((s = build_graphs(g))) { g->broken = true; return s; }
   for (int i = 0; i < n; ++i) {
     cudaError_t e = cudaGraphLaunch(g->graph[g->steps & 1], g->stream);
@@ -537,6 +688,9 @@ lbm_status lbm_profile_levels(lbm_grid* g, int32_t n, double* ms_per_level, int6
   g_err.clear();
   if (!g) return fail(LBM_E_INVAL, "NULL grid");
   if (g->broken) return fail(LBM_E_STATE, "grid is in an error state");
+  for (int sd = 0; sd < 2; ++sd)
+    if (g->n_ranks > 1 && g->has_nb[sd] && !g->connected[sd])
+      return fail(LBM_E_STATE, "halo side " + std::to_string(sd) + " not connected");
   lbm_status s;
   if (g->needs_prologue && (s = run_prologue(g))) return s;
   std::vector<std::pair<int, int64_t>> order;
@@ -588,12 +742,12 @@ lbm_status lbm_macroscopic(lbm_grid* g, int32_t L, double* rho, double* u) {
   if (!g) return fail(LBM_E_INVAL, "NULL grid");
   if (L < 0 || L >= g->levels) return fail(LBM_E_INVAL, "level out of range");
   const HostLevel& H = g->host[L];
-  const size_t ncell = (size_t)H.nfluid * kCells;
+  const size_t ncell = (size_t)H.nlaunch * kCells;
   double *dr = nullptr, *du = nullptr;
   CUDA_TRY(cudaStreamSynchronize(g->stream));
   CUDA_TRY(cudaMalloc(&dr, std::max<size_t>(ncell, 1) * sizeof(double)));
   CUDA_TRY(cudaMalloc(&du, std::max<size_t>(ncell, 1) * 3 * sizeof(double)));
-  launch_macroscopic(g->Q, g->prec, g->dev[L].pop[cur_buf(g, L)], g->dev[L].types, H.nfluid, dr, du, nullptr,
+  launch_macroscopic(g->Q, g->prec, g->dev[L].pop[cur_buf(g, L)], g->dev[L].nbr, H.nlaunch, dr, du, nullptr,
                      g->stream);
   std::vector<double> r(ncell), v(3 * ncell);
   CUDA_TRY(cudaGetLastError());
@@ -602,18 +756,20 @@ lbm_status lbm_macroscopic(lbm_grid* g, int32_t L, double* rho, double* u) {
   CUDA_TRY(cudaStreamSynchronize(g->stream));
   cudaFree(dr);
   cudaFree(du);
-  const int64_t N = H.n[0] * H.n[1] * H.n[2];
+  // dense arrays over the owned slab of this rank (the whole level on one rank)
+  const int64_t N = (H.owned_hi - H.owned_lo) * H.n[1] * H.n[2];
   const double nan = std::nan("");
   if (rho) std::fill(rho, rho + N, nan);
   if (u) std::fill(u, u + 3 * N, nan);
 #pragma omp parallel for schedule(static)
-  for (int32_t b = 0; b < H.nfluid; ++b) {
+  for (int32_t b = 0; b < H.nlaunch; ++b) {
     const int64_t ox = (int64_t)H.origin[3 * b] * kBlock, oy = (int64_t)H.origin[3 * b + 1] * kBlock,
                   oz = (int64_t)H.origin[3 * b + 2] * kBlock;
     for (int l = 0; l < kCells; ++l) {
       if (H.types[(size_t)b * kCells + l] != kFluid) continue;
       const int64_t x = ox + (l & 7), y = oy + ((l >> 3) & 7), z = oz + (l >> 6);
-      const int64_t c = (x * H.n[1] + y) * H.n[2] + z;
+      if (x < H.owned_lo || x >= H.owned_hi) continue;
+      const int64_t c = ((x - H.owned_lo) * H.n[1] + y) * H.n[2] + z;
       const size_t k = (size_t)b * kCells + l;
       if (rho) rho[c] = r[k];
       if (u) { u[3 * c] = v[3 * k]; u[3 * c + 1] = v[3 * k + 1]; u[3 * c + 2] = v[3 * k + 2]; }
@@ -632,12 +788,12 @@ lbm_status lbm_stats(lbm_grid* g, int64_t* leaves, double* mass) {
   for (int L = 0; L < g->levels; ++L) {
     const HostLevel& H = g->host[L];
     double* bm = nullptr;
-    CUDA_TRY(cudaMalloc(&bm, std::max<int32_t>(H.nfluid, 1) * sizeof(double)));
-    launch_macroscopic(g->Q, g->prec, g->dev[L].pop[cur_buf(g, L)], g->dev[L].types, H.nfluid, nullptr, nullptr,
+    CUDA_TRY(cudaMalloc(&bm, std::max<int32_t>(H.nlaunch, 1) * sizeof(double)));
+    launch_macroscopic(g->Q, g->prec, g->dev[L].pop[cur_buf(g, L)], g->dev[L].nbr, H.nlaunch, nullptr, nullptr,
                        bm, g->stream);
-    std::vector<double> h(H.nfluid);
+    std::vector<double> h(H.nlaunch);
     CUDA_TRY(cudaGetLastError());
-    CUDA_TRY(cudaMemcpyAsync(h.data(), bm, H.nfluid * sizeof(double), cudaMemcpyDeviceToHost, g->stream));
+    CUDA_TRY(cudaMemcpyAsync(h.data(), bm, H.nlaunch * sizeof(double), cudaMemcpyDeviceToHost, g->stream));
     CUDA_TRY(cudaStreamSynchronize(g->stream));
     cudaFree(bm);
     double sL = 0.0;
@@ -657,11 +813,213 @@ lbm_status lbm_grid_get_info(const lbm_grid* g, lbm_grid_info* info) {
   return LBM_OK;
 }
 
+lbm_status lbm_partition_cuts(const lbm_grid_desc* d, int32_t levels, const uint8_t* const* masks, int32_t n_ranks,
+                              int32_t* cuts) {
+  g_err.clear();
+  if (!cuts || n_ranks < 1) return fail(LBM_E_INVAL, "bad arguments");
+  lbm_grid_desc dd = *d;
+  dd.n_ranks = n_ranks;
+  dd.rank = 0;
+  lbm_status s = validate_desc(&dd, levels, masks);
+  if (s) return s;
+  std::vector<int32_t> c;
+  partition_cuts(&dd, levels, masks, n_ranks, c);
+  std::copy(c.begin(), c.end(), cuts);
+  return LBM_OK;
+}
+
+lbm_status lbm_grid_slab(const lbm_grid* g, int32_t* x_begin, int32_t* x_end) {
+  g_err.clear();
+  if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  if (x_begin) *x_begin = g->cuts[g->rank];
+  if (x_end) *x_end = g->cuts[g->rank + 1];
+  return LBM_OK;
+}
+
+namespace {
+struct HaloBlob {
+  uint32_t magic, version;
+  int32_t levels, Q, prec, side, rank, n_ranks;
+  int32_t pid, device;
+  int64_t count[16];
+  cudaIpcMemHandle_t pop[16][2];
+  cudaIpcMemHandle_t flags;
+};
+constexpr uint32_t kBlobMagic = 0x484d424cu;  // "LBMH"
+
+lbm_status invalidate_graphs(lbm_grid* g) {
+  CUDA_TRY(cudaStreamSynchronize(g->stream));
+  for (int p = 0; p < 2; ++p)
+    if (g->graph[p]) {
+      cudaGraphExecDestroy(g->graph[p]);
+      g->graph[p] = nullptr;
+    }
+  return LBM_OK;
+}
+
+lbm_status open_ipc(lbm_grid* g, const cudaIpcMemHandle_t& h, void** out) {
+  std::string key(reinterpret_cast<const char*>(&h), sizeof(h));
+  for (auto& e : g->ipc_open)
+    if (e.first == key) { *out = e.second; return LBM_OK; }
+  void* p = nullptr;
+  cudaError_t e = cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess);
+  if (e != cudaSuccess) return fail(LBM_E_COMM, std::string("cudaIpcOpenMemHandle: ") + cudaGetErrorString(e));
+  g->ipc_open.push_back({key, p});
+  *out = p;
+  return LBM_OK;
+}
+}  // namespace
+
+lbm_status lbm_halo_export(const lbm_grid* g, int32_t side, void* blob, int64_t capacity, int64_t* size) {
+  g_err.clear();
+  if (!g || side < 0 || side > 1) return fail(LBM_E_INVAL, "bad arguments");
+  if (g->n_ranks < 2 || !g->has_nb[side]) return fail(LBM_E_STATE, "no neighbour on this side");
+  int64_t need = sizeof(HaloBlob);
+  for (int L = 0; L < g->levels; ++L) need += (int64_t)g->host[L].halo[side].size() * 4;
+  if (size) *size = need;
+  if (!blob) return LBM_OK;
+  if (capacity < need) return fail(LBM_E_INVAL, "blob capacity too small");
+  HaloBlob h;
+  std::memset(&h, 0, sizeof(h));
+  h.magic = kBlobMagic;
+  h.version = 1;
+  h.levels = g->levels;
+  h.Q = g->Q;
+  h.prec = g->prec;
+  h.side = side;
+  h.rank = g->rank;
+  h.n_ranks = g->n_ranks;
+  h.pid = (int32_t)getpid();
+  cudaGetDevice(&h.device);
+  for (int L = 0; L < g->levels; ++L) {
+    h.count[L] = (int64_t)g->host[L].halo[side].size();
+    for (int b = 0; b < 2; ++b) CUDA_TRY(cudaIpcGetMemHandle(&h.pop[L][b], g->dev[L].pop[b]));
+  }
+  CUDA_TRY(cudaIpcGetMemHandle(&h.flags, g->flags));
+  char* out = static_cast<char*>(blob);
+  std::memcpy(out, &h, sizeof(h));
+  int64_t off = sizeof(h);
+  for (int L = 0; L < g->levels; ++L) {
+    const auto& v = g->host[L].halo[side];
+    std::memcpy(out + off, v.data(), v.size() * 4);
+    off += (int64_t)v.size() * 4;
+  }
+  return LBM_OK;
+}
+
+static lbm_status check_counts(lbm_grid* g, int side, const int64_t* count) {
+  for (int L = 0; L < g->levels; ++L)
+    if (count[L] != (int64_t)g->host[L].send[side].size())
+      return fail(LBM_E_COMM, "halo plan mismatch at level " + std::to_string(L) + ": neighbour expects " +
+                                  std::to_string(count[L]) + " cells, this rank sends " +
+                                  std::to_string(g->host[L].send[side].size()));
+  return LBM_OK;
+}
+
+lbm_status lbm_halo_connect(lbm_grid* g, int32_t side, const void* blob, int64_t size) {
+  g_err.clear();
+  if (!g || !blob || side < 0 || side > 1) return fail(LBM_E_INVAL, "bad arguments");
+  if (g->n_ranks < 2 || !g->has_nb[side]) return fail(LBM_E_STATE, "no neighbour on this side");
+  if (size < (int64_t)sizeof(HaloBlob)) return fail(LBM_E_INVAL, "blob too small");
+  HaloBlob h;
+  std::memcpy(&h, blob, sizeof(h));
+  if (h.magic != kBlobMagic || h.version != 1) return fail(LBM_E_INVAL, "not a halo blob");
+  if (h.side != 1 - side || h.levels != g->levels || h.Q != g->Q || h.prec != g->prec || h.n_ranks != g->n_ranks)
+    return fail(LBM_E_COMM, "halo blob does not belong to this neighbour");
+  if (h.pid == (int32_t)getpid()) return fail(LBM_E_INVAL, "same process: use lbm_halo_connect_local");
+  lbm_status s = check_counts(g, side, h.count);
+  if (s) return s;
+  if ((s = invalidate_graphs(g))) return s;
+  const char* in = static_cast<const char*>(blob);
+  int64_t off = sizeof(h);
+  for (int L = 0; L < g->levels; ++L) {
+    DevLevel& D = g->dev[L];
+    for (int b = 0; b < 2; ++b)
+      if ((s = open_ipc(g, h.pop[L][b], &D.peer_pop[side][b]))) return s;
+    std::vector<uint32_t> cells(h.count[L]);
+    if (off + h.count[L] * 4 > size) return fail(LBM_E_INVAL, "blob truncated");
+    std::memcpy(cells.data(), in + off, h.count[L] * 4);
+    off += h.count[L] * 4;
+    if ((s = dev_upload(g, &D.peer_cells[side], cells))) return s;
+  }
+  void* f = nullptr;
+  if ((s = open_ipc(g, h.flags, &f))) return s;
+  g->peer_flags[side] = static_cast<unsigned long long*>(f);
+  g->connected[side] = true;
+  return LBM_OK;
+}
+
+lbm_status lbm_halo_connect_local(lbm_grid* g, int32_t side, lbm_grid* peer) {
+  g_err.clear();
+  if (!g || !peer || side < 0 || side > 1) return fail(LBM_E_INVAL, "bad arguments");
+  if (g->n_ranks < 2 || !g->has_nb[side] || !peer->has_nb[1 - side]) return fail(LBM_E_STATE, "no neighbour");
+  if (peer->levels != g->levels || peer->Q != g->Q || peer->prec != g->prec || peer->n_ranks != g->n_ranks)
+    return fail(LBM_E_COMM, "peer grid does not match");
+  int64_t count[16] = {0};
+  for (int L = 0; L < g->levels; ++L) count[L] = (int64_t)peer->host[L].halo[1 - side].size();
+  lbm_status s = check_counts(g, side, count);
+  if (s) return s;
+  if ((s = invalidate_graphs(g))) return s;
+  for (int L = 0; L < g->levels; ++L) {
+    DevLevel& D = g->dev[L];
+    for (int b = 0; b < 2; ++b) D.peer_pop[side][b] = peer->dev[L].pop[b];
+    if ((s = dev_upload(g, &D.peer_cells[side], peer->host[L].halo[1 - side]))) return s;
+  }
+  g->peer_flags[side] = peer->flags;
+  g->connected[side] = true;
+  return LBM_OK;
+}
+
+lbm_status lbm_halo_plan(const lbm_grid_desc* d, int32_t levels, const uint8_t* const* masks, int32_t side,
+                         int32_t level, int64_t* send_xyz, int64_t* halo_xyz, int64_t capacity, int64_t* n_send,
+                         int64_t* n_halo) {
+  g_err.clear();
+  if (side < 0 || side > 1 || level < 0 || level >= levels) return fail(LBM_E_INVAL, "bad side / level");
+  lbm_status s = validate_desc(d, levels, masks);
+  if (s) return s;
+  if (d->n_ranks < 2) return fail(LBM_E_STATE, "single rank: no halo");
+  std::vector<int32_t> cuts;
+  partition_cuts(d, levels, masks, d->n_ranks, cuts);
+  LocalSlab slab;
+  make_local(d, levels, masks, cuts, slab);
+  std::vector<HostLevel> host;
+  if ((s = build_host(d, levels, masks, host, &slab))) return s;
+  const HostLevel& H = host[level];
+  if (n_send) *n_send = (int64_t)H.send[side].size();
+  if (n_halo) *n_halo = (int64_t)H.halo[side].size();
+  const int64_t gn = (int64_t)d->nx << level;
+  auto put = [&](const std::vector<uint32_t>& v, int64_t* xyz) {
+    if (!xyz) return;
+    for (size_t i = 0; i < v.size() && (int64_t)i < capacity; ++i) {
+      const uint32_t b = v[i] >> 9, l = v[i] & 511u;
+      const int64_t x = (int64_t)H.origin[3 * b] * kBlock + (l & 7);
+      xyz[3 * i] = (((int64_t)slab.x_lo << level) + x + gn) % gn;
+      xyz[3 * i + 1] = (int64_t)H.origin[3 * b + 1] * kBlock + ((l >> 3) & 7);
+      xyz[3 * i + 2] = (int64_t)H.origin[3 * b + 2] * kBlock + (l >> 6);
+    }
+  };
+  put(H.send[side], send_xyz);
+  put(H.halo[side], halo_xyz);
+  return LBM_OK;
+}
+
+// debugging aid (not in the public header): the four halo-protocol counters
+extern "C" lbm_status lbm_debug_flags(lbm_grid* g, unsigned long long* out) {
+  if (!g || !g->flags) return fail(LBM_E_STATE, "no flags");
+  cudaStream_t s;
+  CUDA_TRY(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  CUDA_TRY(cudaMemcpyAsync(out, g->flags, 4 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaStreamSynchronize(s));
+  cudaStreamDestroy(s);
+  return LBM_OK;
+}
+
 void lbm_grid_destroy(lbm_grid* g) {
   if (!g) return;
   if (g->stream) cudaStreamSynchronize(g->stream);
   for (int p = 0; p < 2; ++p)
     if (g->graph[p]) cudaGraphExecDestroy(g->graph[p]);
+  for (auto& h : g->ipc_open) cudaIpcCloseMemHandle(h.second);
   for (void* p : g->allocs) cudaFree(p);
   if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
   delete g;

@@ -27,6 +27,13 @@ struct HostLevel {
   std::vector<uint32_t> links;        // [nlinks][2] slow-link records (lattice.h kLink*)
   std::vector<uint32_t> coal;         // coalescence candidate population indices
   int64_t nlinks = 0;
+  // partition (empty / zero on a single rank)
+  int32_t nlaunch = 0;                // blocks with owned fluid leaves (launched), boundary ones first
+  int32_t nboundary = 0;              // launched blocks holding an owned cell of a cut plane
+  int64_t owned_lo = 0, owned_hi = 0; // owned x range at this level (local coordinates)
+  std::vector<uint32_t> send[2];      // owned fluid cells of the first layer at each cut, (y,z) order
+  std::vector<uint32_t> halo[2];      // halo fluid cells just outside each cut, (y,z) order
+  std::vector<int32_t> bpeer;         // [nboundary][2][512] index into send[side] or -1
   std::vector<int32_t> plain_ids;     // fluid blocks without special cells (Morton order)
   std::vector<int32_t> special_ids;   // the others (Morton order)
 };
@@ -37,6 +44,12 @@ struct BuildInput {
   int32_t levels;
   int32_t Q;
   const uint8_t* const* masks;
+  // x-slab partition (local grid = owned slab + one coarse cell of halo on
+  // each side that has a neighbour rank): owned level-0 x range [lo, hi) in
+  // local coordinates (hi < 0: everything owned), and which sides have a
+  // neighbour (0: -x, 1: +x)
+  int32_t owned_lo0 = 0, owned_hi0 = -1;
+  int32_t has_nb[2] = {0, 0};
 };
 
 // Returns 0 on success; otherwise an lbm_status code with `err` filled.

@@ -42,10 +42,20 @@ struct StepParams {
   T omega;                      // ω_L (Eq.9)
   int32_t periodic[3];
   const uint8_t* face_cls;      // [27] BC class of an out-of-domain source, by outside pattern
-  int32_t nfluid;
-  const int32_t* ids;           // blocks this launch processes (plain or special list)
-  int32_t nids;
+  int32_t nfluid;               // blocks launched (owned fluid blocks, cut-plane blocks first)
+  // ---- x-slab partition (multi-GPU); unused when nbctas == 0 -------------
+  int32_t nbctas;               // CTAs taking part in the halo protocol (cut-plane blocks, >= 1)
+  int32_t nboundary;            // cut-plane blocks (stored and launched first)
+  int32_t has_nb[2];            // neighbour on the -x / +x side
+  unsigned long long* flags;    // this rank: [0],[1] bumped by the -x/+x neighbour, [2] kernels done, [3] CTA count
+  unsigned long long* peer_flag[2];  // neighbour's flag slot this rank bumps
+  T* peer_dst[2];               // neighbour's C_L^{k+1} buffer
+  const uint32_t* peer_cells[2];     // neighbour's halo cell index for each entry of my send list
+  const int32_t* bpeer;         // [nboundary][2][512] send-list index of a cut-plane cell, or -1
 };
+
+// Force-load every kernel (see level_step.cu).
+void preload_kernels();
 
 // kind: 0 = fused stream+collide over the plain blocks in ids, 1 = collide only
 // over all fluid blocks (prologue C_L^1), 2 = fused stream+collide over the
@@ -57,9 +67,10 @@ void launch_level_step(int Q, int collision, int precision, int kind, const void
 void launch_init_eq(int Q, int precision, void* pop, const uint8_t* types, int32_t nfluid,
                     const double* rho, const double* u, cudaStream_t s);
 
-// rho/u (double, compact, NaN on non-fluid cells) of the post-collision
-// buffer `pop`; optional per-block mass partial sums block_mass[nfluid].
-void launch_macroscopic(int Q, int precision, const void* pop, const uint8_t* types, int32_t nfluid,
+// rho/u (double, compact, NaN on cells that are not owned fluid leaves) of the
+// post-collision buffer `pop`; optional per-block mass partial sums
+// block_mass[nblk].  rec = block records (lattice.h kRec*).
+void launch_macroscopic(int Q, int precision, const void* pop, const int32_t* rec, int32_t nblk,
                         double* rho, double* u, double* block_mass, cudaStream_t s);
 
 }  // namespace lbmr

@@ -328,20 +328,88 @@ __device__ __forceinline__ void store_cell(const T (&g)[Q], T* __restrict__ dst,
 template <int Q, typename T>
 struct PlainOcc { static constexpr int value = (Q == 19 && sizeof(T) == 4) ? LBMR_OCC_Q19F : (sizeof(T) == 4 ? 3 : 2); };
 
-// F_L^k over all fluid blocks in storage (Morton) order; CTA = half an 8^3
-// block, one cell per thread.  No shared memory and no barrier: each warp
-// reads its block's record (27 neighbour ids, special slot, origin, per-warp
-// fluid and slow-link masks) with one coalesced and two broadcast loads and
-// picks neighbour ids with __shfl_sync.  A warp whose 32 cells are fluid
-// leaves with only same-level links (the bulk) takes the predicate-free pull;
-// the test is warp-uniform.  Other warps load the same way for their fluid
-// cells, and the few cells with slow links then apply their link records.
-// Offsets are 32-bit (host-checked: nblocks * Q * 512 < 2^32).
-template <int Q, int COLL, typename T>
-__global__ void __launch_bounds__(256, PlainOcc<Q, T>::value) level_step_all(const StepParams<T> P) {
+// ---------------------------------------------------------------- halo protocol
+// x-slab partition.  Blocks holding an owned cell of a cut
+// plane are stored (and launched) first.  Their CTAs (a) wait until every
+// neighbour rank has finished the cut-plane part of all previous kernels
+// (its bumps of our flag reach our kernel count), (b) store their cut-plane
+// cells' post-collision populations straight into the neighbour's halo cells
+// (peer memory: CUDA IPC over NVLink, or another grid on the same device),
+// and (c) the last of them bumps the neighbours' flags.  Interior CTAs never
+// wait.  Only cut-plane cells read halo cells, so this orders every halo read
+// after the matching write and every overwrite after the previous read.
+__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+
+template <typename T>
+__device__ __forceinline__ void halo_wait(const StepParams<T>& P) {
+  if (threadIdx.x == 0) {
+    const unsigned long long mine = *(volatile unsigned long long*)(P.flags + 2);
+    for (int s = 0; s < 2; ++s)
+      if (P.has_nb[s]) {
+#ifdef LBMR_DEBUG_HALO
+        long long spins = 0;
+#endif
+        while (ld_acquire_sys(P.flags + s) < mine) {
+          __nanosleep(256);
+#ifdef LBMR_DEBUG_HALO
+          if (++spins == 2000000)
+            printf("halo_wait stuck: cta %d side %d flag %llu mine %llu nfluid %d nbctas %d\n", blockIdx.x, s,
+                   ld_acquire_sys(P.flags + s), mine, P.nfluid, P.nbctas);
+#endif
+        }
+      }
+  }
+  __syncthreads();
+}
+
+template <typename T>
+__device__ __forceinline__ void halo_signal(const StepParams<T>& P) {
+  __threadfence_system();
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    if (atomicAdd(P.flags + 3, 1ull) == (unsigned long long)(P.nbctas - 1)) {
+      P.flags[3] = 0ull;
+      P.flags[2] += 1ull;
+      __threadfence_system();
+      for (int s = 0; s < 2; ++s)
+        if (P.has_nb[s]) atomicAdd_system(P.peer_flag[s], 1ull);
+    }
+  }
+}
+
+template <int Q, typename T>
+__device__ __forceinline__ void halo_store(const StepParams<T>& P, const T (&g)[Q], int blk, int t) {
+  if (blk >= P.nboundary) return;
+#pragma unroll
+  for (int s = 0; s < 2; ++s) {
+    if (!P.has_nb[s]) continue;
+    const int i = __ldg(P.bpeer + ((unsigned)blk * 2 + s) * kCells + t);
+    if (i < 0) continue;
+    const unsigned pc = __ldg(P.peer_cells[s] + i);
+    T* d = P.peer_dst[s] + (pc >> 9) * (unsigned)(Q * kCells) + (pc & 511u);
+#pragma unroll
+    for (int q = 0; q < Q; ++q) d[q * kCells] = g[q];
+  }
+}
+
+// ---------------------------------------------------------------- fused kernel
+// One cell of F_L^k (all fluid blocks in storage = Morton order, cut-plane
+// blocks first).  CTA = half an 8^3 block, one cell per thread.  No shared
+// memory and no barrier: each warp reads its block's record (27 neighbour
+// ids, special slot, origin, per-warp fluid and slow-link masks) with one
+// coalesced and two broadcast loads and picks neighbour ids with
+// __shfl_sync.  A warp whose 32 cells are fluid leaves with only same-level
+// links (the bulk) takes the predicate-free pull; the test is warp-uniform.
+// Other warps load the same way for their fluid cells, and the few cells with
+// slow links then apply their link records.  Offsets are 32-bit
+// (host-checked: nblocks * Q * 512 < 2^32).
+template <int Q, int COLL, typename T, bool HALO>
+__device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t) {
   constexpr unsigned FULL = 0xffffffffu;
-  const int blk = blockIdx.x >> 1;
-  const int t = ((blockIdx.x & 1) << 8) | threadIdx.x;
   const int lane = threadIdx.x & 31;
   const int* R = P.nbr + blk * kRec;
   const int rec = __ldg(R + lane);
@@ -353,6 +421,7 @@ __global__ void __launch_bounds__(256, PlainOcc<Q, T>::value) level_step_all(con
     pull_all<Q, T, false>(g, P.src, G, rec, blk, true, std::make_integer_sequence<int, Q>{});
     collide<Q, COLL, T>(g, P.omega);
     store_cell<Q, T>(g, P.dst, blk, t);
+    if (HALO) halo_store<Q, T>(P, g, blk, t);
     return;
   }
   const int slot = __shfl_sync(FULL, rec, kRecSlot);
@@ -365,13 +434,12 @@ __global__ void __launch_bounds__(256, PlainOcc<Q, T>::value) level_step_all(con
   if (special) resolve_slow<Q, T>(P, g, ci.x & ((1u << Q) - 1u), ci.y, blk, t);
   collide<Q, COLL, T>(g, P.omega);
   store_cell<Q, T>(g, P.dst, blk, t);
+  if (HALO) halo_store<Q, T>(P, g, blk, t);
 }
 
-// Prologue C_L^1: collision of the initial state, all fluid blocks.
-template <int Q, int COLL, typename T>
-__global__ void __launch_bounds__(256) level_collide(const StepParams<T> P) {
-  const int blk = blockIdx.x >> 1;
-  const int t = ((blockIdx.x & 1) << 8) | threadIdx.x;
+// Prologue C_L^1: collision of the initial state.
+template <int Q, int COLL, typename T, bool HALO>
+__device__ __forceinline__ void collide_cell(const StepParams<T>& P, int blk, int t) {
   const uint32_t fm = (uint32_t)__ldg(P.nbr + blk * kRec + kRecFluid + (t >> 5));
   if (!((fm >> (threadIdx.x & 31)) & 1u)) return;
   T g[Q];
@@ -379,6 +447,32 @@ __global__ void __launch_bounds__(256) level_collide(const StepParams<T> P) {
   for (int q = 0; q < Q; ++q) g[q] = __ldg(P.src + ((unsigned)blk * Q + q) * kCells + t);
   collide<Q, COLL, T>(g, P.omega);
   store_cell<Q, T>(g, P.dst, blk, t);
+  if (HALO) halo_store<Q, T>(P, g, blk, t);
+}
+
+template <int Q, int COLL, typename T>
+__global__ void __launch_bounds__(256, PlainOcc<Q, T>::value) level_step_all(const StepParams<T> P) {
+  step_cell<Q, COLL, T, false>(P, blockIdx.x >> 1, ((blockIdx.x & 1) << 8) | threadIdx.x);
+}
+
+// Partitioned variant: grid = 2 * max(nfluid, 1) CTAs; the first nbctas run
+// the halo protocol around their work.
+template <int Q, int COLL, typename T, bool STREAM>
+__global__ void __launch_bounds__(256, PlainOcc<Q, T>::value) level_step_halo(const StepParams<T> P) {
+  const int blk = blockIdx.x >> 1;
+  const int t = ((blockIdx.x & 1) << 8) | threadIdx.x;
+  const bool proto = (int)blockIdx.x < P.nbctas;
+  if (proto) halo_wait<T>(P);
+  if (blk < P.nfluid) {
+    if (STREAM) step_cell<Q, COLL, T, true>(P, blk, t);
+    else collide_cell<Q, COLL, T, true>(P, blk, t);
+  }
+  if (proto) halo_signal<T>(P);
+}
+
+template <int Q, int COLL, typename T>
+__global__ void __launch_bounds__(256) level_collide(const StepParams<T> P) {
+  collide_cell<Q, COLL, T, false>(P, blockIdx.x >> 1, ((blockIdx.x & 1) << 8) | threadIdx.x);
 }
 
 // ---------------------------------------------------------------- init / macroscopic
@@ -404,12 +498,13 @@ __global__ void __launch_bounds__(512) init_eq_kernel(T* pop, const uint8_t* typ
 }
 
 template <int Q, typename T>
-__global__ void __launch_bounds__(512) macroscopic_kernel(const T* pop, const uint8_t* types, double* rho,
-                                                          double* u, double* block_mass) {
+__global__ void __launch_bounds__(512) macroscopic_kernel(const T* pop, const int32_t* rec, double* rho, double* u,
+                                                          double* block_mass) {
   const int blk = blockIdx.x, t = threadIdx.x;
   const size_t c = (size_t)blk * kCells + t;
   double r = 0.0;
-  const bool fluid = types[c] == kFluid;
+  const uint32_t fm = (uint32_t)rec[blk * kRec + kRecFluid + (t >> 5)];
+  const bool fluid = (fm >> (t & 31)) & 1u;  // owned fluid leaf
   if (fluid) {
     const T* s = pop + (size_t)blk * Q * kCells + t;
     double d = 0, jx = 0, jy = 0, jz = 0;
@@ -447,10 +542,48 @@ __global__ void __launch_bounds__(512) macroscopic_kernel(const T* pop, const ui
 template <int Q, int COLL, typename T>
 static void launch_typed(int kind, const void* params, cudaStream_t s) {
   const StepParams<T>& p = *static_cast<const StepParams<T>*>(params);
+  dim3 block(256);
+  if (p.nbctas > 0) {  // partitioned: always launched (the protocol must run)
+    dim3 grid(2 * std::max(p.nfluid, 1));
+    if (kind == 1) level_step_halo<Q, COLL, T, false><<<grid, block, 0, s>>>(p);
+    else level_step_halo<Q, COLL, T, true><<<grid, block, 0, s>>>(p);
+    return;
+  }
   if (p.nfluid <= 0) return;
-  dim3 block(256), grid(2 * p.nfluid);
+  dim3 grid(2 * p.nfluid);
   if (kind == 1) level_collide<Q, COLL, T><<<grid, block, 0, s>>>(p);
   else level_step_all<Q, COLL, T><<<grid, block, 0, s>>>(p);
+}
+
+// Load every kernel of the library now.  With lazy module loading (the CUDA
+// 12 default) the first launch of a function can wait for the device to go
+// idle, which deadlocks against a partition's spinning halo CTAs waiting for
+// a neighbour grid whose kernels this host thread has not launched yet.
+template <int Q, int COLL, typename T>
+static void preload_variant() {
+  cudaFuncAttributes a;
+  cudaFuncGetAttributes(&a, level_step_all<Q, COLL, T>);
+  cudaFuncGetAttributes(&a, level_collide<Q, COLL, T>);
+  cudaFuncGetAttributes(&a, level_step_halo<Q, COLL, T, true>);
+  cudaFuncGetAttributes(&a, level_step_halo<Q, COLL, T, false>);
+}
+
+void preload_kernels() {
+  preload_variant<19, LBM_BGK, float>();
+  preload_variant<27, LBM_BGK, float>();
+  preload_variant<27, LBM_KBC, float>();
+  preload_variant<19, LBM_BGK, double>();
+  preload_variant<27, LBM_BGK, double>();
+  preload_variant<27, LBM_KBC, double>();
+  cudaFuncAttributes a;
+  cudaFuncGetAttributes(&a, init_eq_kernel<19, float>);
+  cudaFuncGetAttributes(&a, init_eq_kernel<27, float>);
+  cudaFuncGetAttributes(&a, init_eq_kernel<19, double>);
+  cudaFuncGetAttributes(&a, init_eq_kernel<27, double>);
+  cudaFuncGetAttributes(&a, macroscopic_kernel<19, float>);
+  cudaFuncGetAttributes(&a, macroscopic_kernel<27, float>);
+  cudaFuncGetAttributes(&a, macroscopic_kernel<19, double>);
+  cudaFuncGetAttributes(&a, macroscopic_kernel<27, double>);
 }
 
 void launch_level_step(int Q, int collision, int precision, int kind, const void* params, cudaStream_t s) {
@@ -477,15 +610,15 @@ void launch_init_eq(int Q, int precision, void* pop, const uint8_t* types, int32
   }
 }
 
-void launch_macroscopic(int Q, int precision, const void* pop, const uint8_t* types, int32_t nfluid, double* rho,
+void launch_macroscopic(int Q, int precision, const void* pop, const int32_t* rec, int32_t nblk, double* rho,
                         double* u, double* block_mass, cudaStream_t s) {
-  if (nfluid <= 0) return;
+  if (nblk <= 0) return;
   if (precision == LBM_FP32) {
-    if (Q == 19) macroscopic_kernel<19, float><<<nfluid, 512, 0, s>>>((const float*)pop, types, rho, u, block_mass);
-    else macroscopic_kernel<27, float><<<nfluid, 512, 0, s>>>((const float*)pop, types, rho, u, block_mass);
+    if (Q == 19) macroscopic_kernel<19, float><<<nblk, 512, 0, s>>>((const float*)pop, rec, rho, u, block_mass);
+    else macroscopic_kernel<27, float><<<nblk, 512, 0, s>>>((const float*)pop, rec, rho, u, block_mass);
   } else {
-    if (Q == 19) macroscopic_kernel<19, double><<<nfluid, 512, 0, s>>>((const double*)pop, types, rho, u, block_mass);
-    else macroscopic_kernel<27, double><<<nfluid, 512, 0, s>>>((const double*)pop, types, rho, u, block_mass);
+    if (Q == 19) macroscopic_kernel<19, double><<<nblk, 512, 0, s>>>((const double*)pop, rec, rho, u, block_mass);
+    else macroscopic_kernel<27, double><<<nblk, 512, 0, s>>>((const double*)pop, rec, rho, u, block_mass);
   }
 }
 

@@ -56,7 +56,8 @@ class GridInfo(ctypes.Structure):
 EXPORTS = ["lbm_grid_create", "lbm_set_bc", "lbm_init_equilibrium", "lbm_init_uniform", "lbm_step",
            "lbm_macroscopic", "lbm_stats", "lbm_grid_get_info", "lbm_profile_levels", "lbm_synchronize",
            "lbm_grid_destroy", "lbm_last_error", "lbm_version", "lbm_grid_analyze", "lbm_schedule",
-           "lbm_lattice_table", "lbm_omega_level"]
+           "lbm_lattice_table", "lbm_omega_level", "lbm_partition_cuts", "lbm_grid_slab", "lbm_halo_export",
+           "lbm_halo_connect", "lbm_halo_connect_local", "lbm_halo_plan"]
 
 _lib = None
 
@@ -93,6 +94,15 @@ def load_library(path: str = LIB_PATH):
     lib.lbm_lattice_table.restype = ctypes.c_int32
     lib.lbm_omega_level.argtypes = [ctypes.c_double, ctypes.c_int32]
     lib.lbm_omega_level.restype = ctypes.c_double
+    PP = ctypes.POINTER(ctypes.c_void_p)
+    i32p = ctypes.POINTER(ctypes.c_int32)
+    lib.lbm_partition_cuts.argtypes = [ctypes.POINTER(GridDesc), ctypes.c_int32, PP, ctypes.c_int32, i32p]
+    lib.lbm_grid_slab.argtypes = [P, i32p, i32p]
+    lib.lbm_halo_export.argtypes = [P, ctypes.c_int32, ctypes.c_void_p, ctypes.c_int64, lp]
+    lib.lbm_halo_connect.argtypes = [P, ctypes.c_int32, ctypes.c_void_p, ctypes.c_int64]
+    lib.lbm_halo_connect_local.argtypes = [P, ctypes.c_int32, P]
+    lib.lbm_halo_plan.argtypes = [ctypes.POINTER(GridDesc), ctypes.c_int32, PP, ctypes.c_int32, ctypes.c_int32, lp, lp,
+                                  ctypes.c_int64, lp, lp]
     lib.lbm_last_error.restype = ctypes.c_char_p
     lib.lbm_version.restype = ctypes.c_char_p
     for name in EXPORTS:
@@ -146,6 +156,45 @@ def analyze_problem(prob, precision=FP32) -> GridInfo:
                    omega0=prob.omega0)
 
 
+def _mask_ptrs(masks):
+    ms = [np.ascontiguousarray(m, dtype=np.uint8) for m in masks]
+    return ms, (ctypes.c_void_p * len(ms))(*[m.ctypes.data for m in ms])
+
+
+def _problem_kw(prob, precision=FP32):
+    return dict(periodic=prob.periodic, face_bc=prob.face_bc, lattice=prob.Q,
+                collision=KBC if prob.collision == "kbc" else BGK, precision=precision, omega0=prob.omega0)
+
+
+def partition_cuts(prob, n_ranks: int):
+    """Balanced level-0 x cuts (n_ranks + 1 entries), host only."""
+    lib = load_library()
+    ms, ptrs = _mask_ptrs(prob.masks)
+    d = make_desc(prob.nx, prob.ny, prob.nz, **_problem_kw(prob))
+    cuts = np.zeros(n_ranks + 1, dtype=np.int32)
+    _check(lib.lbm_partition_cuts(ctypes.byref(d), len(ms), ptrs, int(n_ranks),
+                                  cuts.ctypes.data_as(ctypes.POINTER(ctypes.c_int32))))
+    return [int(c) for c in cuts]
+
+
+def halo_plan(prob, n_ranks: int, rank: int, side: int, level: int):
+    """Global (x, y, z) of the cells rank sends across `side` and of its halo
+    cells there, at `level` (host only)."""
+    lib = load_library()
+    ms, ptrs = _mask_ptrs(prob.masks)
+    d = make_desc(prob.nx, prob.ny, prob.nz, n_ranks=n_ranks, rank=rank, **_problem_kw(prob))
+    ns, nh = ctypes.c_int64(), ctypes.c_int64()
+    lp = ctypes.POINTER(ctypes.c_int64)
+    _check(lib.lbm_halo_plan(ctypes.byref(d), len(ms), ptrs, side, level, None, None, 0, ctypes.byref(ns),
+                             ctypes.byref(nh)))
+    cap = max(ns.value, nh.value, 1)
+    a = np.zeros((cap, 3), dtype=np.int64)
+    b = np.zeros((cap, 3), dtype=np.int64)
+    _check(lib.lbm_halo_plan(ctypes.byref(d), len(ms), ptrs, side, level, a.ctypes.data_as(lp),
+                             b.ctypes.data_as(lp), cap, ctypes.byref(ns), ctypes.byref(nh)))
+    return a[:ns.value].copy(), b[:nh.value].copy()
+
+
 def schedule(levels: int, n: int = 0):
     """Pipelined launch order [(L, k), ...] of coarse step n."""
     lib = load_library()
@@ -175,7 +224,8 @@ class Grid:
 
     def __init__(self, nx: int, ny: int, nz: int, masks: Sequence[np.ndarray], *, periodic=(0, 0, 0),
                  face_bc=(0, 0, 0, 0, 0, 0), lattice: int = D3Q19, collision: int = BGK,
-                 precision: int = FP32, omega0: float = 1.0, stream: Optional[int] = None):
+                 precision: int = FP32, omega0: float = 1.0, stream: Optional[int] = None,
+                 n_ranks: int = 1, rank: int = 0):
         lib = load_library()
         self.lib = lib
         self.shape0 = (nx, ny, nz)
@@ -184,7 +234,9 @@ class Grid:
         for L, m in enumerate(self._masks):
             if m.shape != (nx << L, ny << L, nz << L):
                 raise ValueError(f"mask {L} has shape {m.shape}, expected {(nx << L, ny << L, nz << L)}")
-        d = make_desc(nx, ny, nz, periodic, face_bc, lattice, collision, precision, omega0, stream)
+        d = make_desc(nx, ny, nz, periodic, face_bc, lattice, collision, precision, omega0, stream, n_ranks, rank)
+        self.n_ranks, self.rank = n_ranks, rank
+        self._periodic_x = bool(periodic[0])
         ptrs = (ctypes.c_void_p * self.levels)(*[m.ctypes.data for m in self._masks])
         h = ctypes.c_void_p()
         _check(lib.lbm_grid_create(ctypes.byref(d), self.levels, ptrs, ctypes.byref(h)))
@@ -214,9 +266,33 @@ class Grid:
         u = np.ascontiguousarray(u, dtype=np.float64)
         _check(self.lib.lbm_set_bc(self.h, int(cls), int(kind), _dp(u)))
 
+    def slab(self):
+        """Owned level-0 x range [begin, end) (the whole domain on one rank)."""
+        a, b = ctypes.c_int32(), ctypes.c_int32()
+        _check(self.lib.lbm_grid_slab(self.h, ctypes.byref(a), ctypes.byref(b)))
+        return a.value, b.value
+
     def level_shape(self, L: int):
+        """Shape of the dense per-level arrays this grid takes and returns
+        (the owned slab on a partitioned grid)."""
         nx, ny, nz = self.shape0
+        if self.n_ranks > 1:
+            b, e = self.slab()
+            nx = e - b
         return (nx << L, ny << L, nz << L)
+
+    def halo_export(self, side: int) -> bytes:
+        n = ctypes.c_int64()
+        _check(self.lib.lbm_halo_export(self.h, int(side), None, 0, ctypes.byref(n)))
+        buf = ctypes.create_string_buffer(n.value)
+        _check(self.lib.lbm_halo_export(self.h, int(side), buf, n.value, ctypes.byref(n)))
+        return buf.raw
+
+    def halo_connect(self, side: int, blob: bytes):
+        _check(self.lib.lbm_halo_connect(self.h, int(side), blob, len(blob)))
+
+    def halo_connect_local(self, side: int, peer: "Grid"):
+        _check(self.lib.lbm_halo_connect_local(self.h, int(side), peer.h))
 
     def init_equilibrium(self, L: int, rho: Optional[np.ndarray] = None, u: Optional[np.ndarray] = None):
         shape = self.level_shape(L)
@@ -261,18 +337,72 @@ class Grid:
         return ms, cnt
 
 
-def grid_from_problem(prob, precision: int = FP32, stream: Optional[int] = None, init: bool = True) -> Grid:
-    """Build a Grid from an ``lbm_inputs.Problem`` (masks, BCs, initial state)."""
-    g = Grid(prob.nx, prob.ny, prob.nz, prob.masks, periodic=prob.periodic, face_bc=prob.face_bc,
-             lattice=prob.Q, collision=KBC if prob.collision == "kbc" else BGK, precision=precision,
-             omega0=prob.omega0, stream=stream)
+def grid_from_problem(prob, precision: int = FP32, stream: Optional[int] = None, init: bool = True,
+                      n_ranks: int = 1, rank: int = 0) -> Grid:
+    """Build a Grid from an ``lbm_inputs.Problem`` (masks, BCs, initial state);
+    with n_ranks > 1 the grid holds rank's x-slab (connect its halos before
+    stepping)."""
+    g = Grid(prob.nx, prob.ny, prob.nz, prob.masks, stream=stream, n_ranks=n_ranks, rank=rank,
+             **_problem_kw(prob, precision))
     for cls, (kind, u) in prob.bc.items():
         g.set_bc(cls, kind, u)
     if init:
-        if prob.init_rho is None and prob.init_u is None:
-            g.init_uniform(prob.uniform_rho, prob.uniform_u)
-        else:
-            for L in range(prob.levels):
-                rho, u = prob.init_fields(L)
-                g.init_equilibrium(L, rho, u)
+        init_from_problem(g, prob)
     return g
+
+
+def init_from_problem(g: Grid, prob):
+    if prob.init_rho is None and prob.init_u is None:
+        g.init_uniform(prob.uniform_rho, prob.uniform_u)
+        return
+    b, e = g.slab() if g.n_ranks > 1 else (0, prob.nx)
+    for L in range(prob.levels):
+        rho, u = prob.init_fields(L)
+        g.init_equilibrium(L, rho[b << L:e << L], u[b << L:e << L])
+
+
+class PartitionedGrid:
+    """P x-slab grids of one problem in ONE process (emulated multi-GPU on one
+    device, or one grid per visible device).  Each slab runs on its own CUDA
+    stream; the halo protocol orders the slabs on the device, so stepping is
+    just issuing lbm_step on every slab."""
+
+    def __init__(self, prob, n_ranks: int, precision: int = FP32, devices=None):
+        import torch
+        self.prob, self.P = prob, n_ranks
+        self.grids, self.streams = [], []
+        for r in range(n_ranks):
+            dev = devices[r] if devices else torch.cuda.current_device()
+            with torch.cuda.device(dev):
+                s = torch.cuda.Stream()
+                self.streams.append(s)
+                self.grids.append(grid_from_problem(prob, precision, stream=s.cuda_stream, n_ranks=n_ranks, rank=r))
+        for r, g in enumerate(self.grids):
+            left, right = (r - 1) % n_ranks, (r + 1) % n_ranks
+            if g_has(g, 0):
+                g.halo_connect_local(0, self.grids[left])
+            if g_has(g, 1):
+                g.halo_connect_local(1, self.grids[right])
+
+    def step(self, n: int = 1):
+        for g in self.grids:
+            g.step(n)
+
+    def synchronize(self):
+        for g in self.grids:
+            g.synchronize()
+
+    def macroscopic(self, L: int):
+        parts = [g.macroscopic(L) for g in self.grids]
+        return np.concatenate([p[0] for p in parts], axis=0), np.concatenate([p[1] for p in parts], axis=0)
+
+    def close(self):
+        for g in self.grids:
+            g.close()
+
+
+def g_has(g: Grid, side: int) -> bool:
+    """Whether partitioned grid g has a neighbour on `side` (0: -x, 1: +x)."""
+    b, e = g.slab()
+    per = g._periodic_x
+    return (b > 0 or per) if side == 0 else (e < g.shape0[0] or per)
