@@ -178,10 +178,16 @@ def main():
         return
 
     import torch
-    torch.cuda.set_device(local)
+    # LBMR_BENCH_SHARE_DEVICE=1: every rank on cuda:0 with gloo (exercises the
+    # N>1 code path on a one-GPU box; its timing is not a scaling number)
+    share = os.environ.get("LBMR_BENCH_SHARE_DEVICE") == "1"
+    torch.cuda.set_device(0 if share else local)
     if ws > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if share:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     from paper_conf_ipps_mahmoudsm24_b200 import lbmr
 
     build_fn, desc = CONFIGS[args.config]
@@ -189,12 +195,26 @@ def main():
     prec = lbmr.FP32 if args.precision == "fp32" else lbmr.FP64
     stream = torch.cuda.Stream()
     t0 = time.perf_counter()
-    g = lbmr.grid_from_problem(prob, precision=prec, stream=stream.cuda_stream, init=False)
-    g.init_uniform(prob.uniform_rho, prob.uniform_u) if prob.init_u is None else [
-        g.init_equilibrium(L, *prob.init_fields(L)) for L in range(prob.levels)]
+    # N > 1: rank's x-slab of the SAME workload (strong scaling), halos written
+    # into the neighbour GPUs' buffers by the level kernels (CUDA IPC / NVLink)
+    g = lbmr.grid_from_problem(prob, precision=prec, stream=stream.cuda_stream, init=False, n_ranks=ws, rank=rank)
+    if ws > 1:
+        import torch.distributed as dist
+        blobs = {side: (g.halo_export(side) if lbmr.g_has(g, side) else None) for side in (0, 1)}
+        allb = [None] * ws
+        dist.all_gather_object(allb, blobs)
+        for side in (0, 1):
+            if lbmr.g_has(g, side):
+                g.halo_connect(side, allb[(rank + (1 if side else -1)) % ws][1 - side])
+    lbmr.init_from_problem(g, prob)
     setup_s = time.perf_counter() - t0
     info = g.info()
-    leaves = [int(info.leaves[L]) for L in range(prob.levels)]
+    leaves_local = [int(info.leaves[L]) for L in range(prob.levels)]
+    leaves = list(leaves_local)
+    if ws > 1:
+        t = torch.tensor(leaves, device="cpu" if share else "cuda", dtype=torch.int64)
+        torch.distributed.all_reduce(t)
+        leaves = [int(v) for v in t.tolist()]
     upd = updates_per_step(leaves)
     kernels_per_step = int(info.kernels_per_step)
 
@@ -205,7 +225,7 @@ def main():
         if ws > 1:
             torch.distributed.barrier()
 
-    sampler = ClockSampler(local)
+    sampler = ClockSampler(0 if share else local)
     sampler.start()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     barrier()
@@ -218,10 +238,10 @@ def main():
     clocks = sampler.stop()
     ms = ev0.elapsed_time(ev1)
     if ws > 1:
-        t = torch.tensor([ms], device="cuda", dtype=torch.float64)
+        t = torch.tensor([ms], device="cpu" if share else "cuda", dtype=torch.float64)
         torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
         ms = float(t.item())
-    value = upd * args.steps * ws / (ms * 1e3)
+    value = upd * args.steps / (ms * 1e3)  # all ranks' updates / max-over-ranks time
 
     # per-level device time (instrumented launches, CUDA events on the same stream)
     ms_lvl, cnt_lvl = g.profile_levels(args.profile_steps)
@@ -229,13 +249,13 @@ def main():
     bpu = 2 * prob.Q * tsz
     dom = int(np.argmax(ms_lvl))
     per_launch_ms = ms_lvl[dom] / max(cnt_lvl[dom], 1)
-    achieved = leaves[dom] * bpu / (per_launch_ms * 1e-3) / 1e9
+    achieved = leaves_local[dom] * bpu / (per_launch_ms * 1e-3) / 1e9
     peak, peak_src = peak_hbm()
     per_level = []
     for L in range(prob.levels):
         pl = ms_lvl[L] / max(cnt_lvl[L], 1)
-        gbs = leaves[L] * bpu / (pl * 1e-3) / 1e9 if pl > 0 else None
-        per_level.append({"level": L, "leaves": leaves[L], "launches": int(cnt_lvl[L]), "ms_per_launch": pl,
+        gbs = leaves_local[L] * bpu / (pl * 1e-3) / 1e9 if pl > 0 else None
+        per_level.append({"level": L, "leaves": leaves_local[L], "launches": int(cnt_lvl[L]), "ms_per_launch": pl,
                           "GBs": gbs, "frac": gbs / peak if gbs else None,
                           "share_of_step": ms_lvl[L] / max(ms_lvl.sum(), 1e-12)})
     traffic = None
@@ -259,12 +279,15 @@ def main():
         g.set_bc(I.CLS_LID, lbmr.BC_VELOCITY, u_in)
         g.step(1)
         _, mass = g.stats()
+        if ws > 1:
+            mt = torch.tensor([mass], device="cpu" if share else "cuda", dtype=torch.float64)
+            torch.distributed.all_reduce(mt)
     e2e_s = time.perf_counter() - t0
     if ws > 1:
-        t = torch.tensor([e2e_s], device="cuda", dtype=torch.float64)
+        t = torch.tensor([e2e_s], device="cpu" if share else "cuda", dtype=torch.float64)
         torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
         e2e_s = float(t.item())
-    e2e = {"value": upd * n_e2e * ws / (e2e_s * 1e6), "unit": "MLUPS",
+    e2e = {"value": upd * n_e2e / (e2e_s * 1e6), "unit": "MLUPS",
            "h2d_bytes_per_step": 32 + 27,
            "d2h_bytes_per_step": 8 * int(sum(info.blocks[L] for L in range(prob.levels))),
            "steps": n_e2e, "what": "per step: lbm_set_bc (H2D) + lbm_step(1) + lbm_stats mass (D2H), wall clock"}
@@ -280,16 +303,17 @@ def main():
         line = {
             "metric": METRIC, "value": value, "unit": "MLUPS", "n_gpus": ws, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
-            "scaling": "weak" if ws > 1 else "strong", "vs_baseline": None,
+            "scaling": "strong", "vs_baseline": None,
             "dtype": "f32" if prec == lbmr.FP32 else "f64", "data": "synthetic",
             "config": {"workload": desc, "levels": prob.levels, "leaves": leaves, "updates_per_step": upd,
-                       "parallelism": "replicas" if ws > 1 else "single",
+                       "parallelism": f"x-slabs x{ws} (halo peer stores over NVLink)" if ws > 1 else "single",
                        "l2": f"working set {dev_bytes / 1e9:.2f} GB > 126 MB L2 (no flush needed)",
                        "precision": args.precision, "setup_s": round(setup_s, 2)},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "kernel": f"level_step L{dom}",
                          "bytes_per_update": bpu, "peak_source": peak_src,
-                         "step_frac": value * 1e6 / ws * bpu / 1e9 / peak},
+                         "step_frac": value * 1e6 / ws * bpu / 1e9 / peak,
+                         "note": "achieved / per_level are this rank's (rank 0) kernels" if ws > 1 else None},
             "per_level": per_level,
             "cpu_baseline": cpu,
             "e2e": e2e,
