@@ -37,6 +37,7 @@ CONFIGS = {
     "tunnel4": (lambda: I.tunnel4(), "cfg5 tunnel4: D3Q19 BGK, 4 levels, 200x105x105 coarse (1600x840x840 eff.)"),
     "sphere3": (lambda: I.sphere3(), "cfg3 sphere3: D3Q19 BGK, 3 levels, 256x128x128 coarse, Re=3700"),
     "cavity4_kbc": (lambda: I.cavity4_kbc(), "cfg4 cavity4: D3Q27 KBC, 4 levels, 384^3 effective"),
+    "cavity4_bgk": (lambda: I.cavity4_kbc(collision="bgk"), "cfg4 geometry with D3Q27 BGK (KBC cost reference)"),
     "uniform512": (lambda: I.uniform(512), "cfg2 uniform512: D3Q19 BGK, single level 512^3 periodic"),
     "cavity2": (lambda: I.cavity2(), "cfg1 cavity2: D3Q19 BGK, 2 levels, 32^3 coarse"),
 }
@@ -45,6 +46,7 @@ REF_SAMPLE = {
     "tunnel4": (lambda: I.tunnel4(scale=5), "tunnel4 geometry at 1/5 scale (40x21x21 coarse, 4 levels)"),
     "sphere3": (lambda: I.sphere3(scale=4), "sphere3 geometry at 1/4 scale (64x32x32 coarse, 3 levels)"),
     "cavity4_kbc": (lambda: I.cavity4_kbc("mini"), "cavity4 KBC at 16^3 coarse, 4 levels"),
+    "cavity4_bgk": (lambda: I.cavity4_kbc("mini", collision="bgk"), "cavity4 geometry D3Q27 BGK at 16^3 coarse"),
     "uniform512": (lambda: I.uniform(64), "uniform periodic 64^3"),
     "cavity2": (lambda: I.cavity2(), "cavity2 (full size)"),
 }

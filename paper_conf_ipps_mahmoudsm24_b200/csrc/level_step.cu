@@ -129,26 +129,59 @@ __device__ __forceinline__ void collide_bgk(T (&g)[Q], T omega) {
 }
 
 // KBC (reading R-A9) on shifted populations; D3Q27 only.
+//   f^neq = g - g^eq;  Δs from the deviatoric second moments of f^neq;
+//   Δh = f^neq - Δs;  γ = 1/β - (2 - 1/β) <Δs|Δh>/<Δh|Δh>,  <X|Y> = Σ X Y / f^eq;
+//   f* = f - β (2 Δs + γ Δh),  β = ω/2.
+// Organised for the ALU: g^eq by opposite pairs (shared even part), second
+// moments from pair sums (e_a e_b is even), one rounded reciprocal per f^eq.
+template <>
+__device__ __forceinline__ double recip<double>(double x) {
+  return __drcp_rn(x);
+}
+
 template <typename T>
 __device__ __forceinline__ void collide_kbc(T (&g)[27], T omega) {
   constexpr int Q = 27;
-  T drho, jx, jy, jz;
-  moments<Q, T>(g, drho, jx, jy, jz);
-  const T rho = T(1) + drho;
-  const T inv = T(1) / rho;
-  const T ux = jx * inv, uy = jy * inv, uz = jz * inv;
-  const T usq15 = T(1.5) * (ux * ux + uy * uy + uz * uz);
-  // g <- f^neq = g - g^eq ; second moments of f^neq
-  T pxx = 0, pyy = 0, pzz = 0, pxy = 0, pxz = 0, pyz = 0;
+  T drho = g[0], jx = T(0), jy = T(0), jz = T(0);
 #pragma unroll
-  for (int q = 0; q < Q; ++q) {
-    g[q] -= geq<Q, T>(q, drho, rho, ux, uy, uz, usq15);
-    if (ex(q)) pxx += g[q];
-    if (ey(q)) pyy += g[q];
-    if (ez(q)) pzz += g[q];
-    if (ex(q) * ey(q) > 0) pxy += g[q]; else if (ex(q) * ey(q) < 0) pxy -= g[q];
-    if (ex(q) * ez(q) > 0) pxz += g[q]; else if (ex(q) * ez(q) < 0) pxz -= g[q];
-    if (ey(q) * ez(q) > 0) pyz += g[q]; else if (ey(q) * ez(q) < 0) pyz -= g[q];
+  for (int q = 1; q < Q; q += 2) {
+    const T sm = g[q] + g[q + 1];
+    const T df = g[q] - g[q + 1];
+    drho += sm;
+    if (ex(q) > 0) jx += df; else if (ex(q) < 0) jx -= df;
+    if (ey(q) > 0) jy += df; else if (ey(q) < 0) jy -= df;
+    if (ez(q) > 0) jz += df; else if (ez(q) < 0) jz -= df;
+  }
+  const T inv = recip<T>(T(1) + drho);
+  const T base = drho - T(1.5) * (jx * jx + jy * jy + jz * jz) * inv;  // g^eq = w (base + 3 e.j + 4.5 (e.j)^2 / rho)
+  const T c45 = T(4.5) * inv;
+  T geq[Q];
+  geq[0] = T(weight<Q>(0)) * base;
+#pragma unroll
+  for (int q = 1; q < Q; q += 2) {
+    T ej = T(0);
+    if (ex(q) > 0) ej += jx; else if (ex(q) < 0) ej -= jx;
+    if (ey(q) > 0) ej += jy; else if (ey(q) < 0) ej -= jy;
+    if (ez(q) > 0) ej += jz; else if (ez(q) < 0) ej -= jz;
+    const T w = T(weight<Q>(q));
+    const T sym = w * (base + c45 * ej * ej);
+    const T asym = w * T(3) * ej;
+    geq[q] = sym + asym;
+    geq[q + 1] = sym - asym;
+  }
+  T pxx = 0, pyy = 0, pzz = 0, pxy = 0, pxz = 0, pyz = 0;
+  g[0] -= geq[0];
+#pragma unroll
+  for (int q = 1; q < Q; q += 2) {
+    g[q] -= geq[q];
+    g[q + 1] -= geq[q + 1];
+    const T ps = g[q] + g[q + 1];
+    if (ex(q)) pxx += ps;
+    if (ey(q)) pyy += ps;
+    if (ez(q)) pzz += ps;
+    if (ex(q) * ey(q) > 0) pxy += ps; else if (ex(q) * ey(q) < 0) pxy -= ps;
+    if (ex(q) * ez(q) > 0) pxz += ps; else if (ex(q) * ez(q) < 0) pxz -= ps;
+    if (ey(q) * ez(q) > 0) pyz += ps; else if (ey(q) * ez(q) < 0) pyz -= ps;
   }
   const T nxz = pxx - pzz, nyz = pyy - pzz;
   const T sx = (T(2) * nxz - nyz) / T(6), sy = (-nxz + T(2) * nyz) / T(6), sz = (-nxz - nyz) / T(6);
@@ -166,11 +199,11 @@ __device__ __forceinline__ void collide_kbc(T (&g)[27], T omega) {
   T sh = 0, hh = 0;
 #pragma unroll
   for (int q = 0; q < Q; ++q) {
-    const T feq = T(weight<Q>(q)) + geq<Q, T>(q, drho, rho, ux, uy, uz, usq15);
+    const T ifeq = recip<T>(T(weight<Q>(q)) + geq[q]);
     const T s = ds(q);
     const T h = g[q] - s;
-    sh += s * h / feq;
-    hh += h * h / feq;
+    sh += s * h * ifeq;
+    hh += h * h * ifeq;
   }
   const T beta = omega / T(2);
   const T gamma = (hh < T(1e-30)) ? T(2) : T(1) / beta - (T(2) - T(1) / beta) * sh / hh;
@@ -178,8 +211,7 @@ __device__ __forceinline__ void collide_kbc(T (&g)[27], T omega) {
   for (int q = 0; q < Q; ++q) {
     const T s = ds(q);
     const T h = g[q] - s;
-    const T e = geq<Q, T>(q, drho, rho, ux, uy, uz, usq15);
-    g[q] = (g[q] + e) - beta * (T(2) * s + gamma * h);
+    g[q] = (geq[q] + g[q]) - beta * (T(2) * s + gamma * h);
   }
 }
 
@@ -292,6 +324,52 @@ struct PullGeom {
   }
 };
 
+// Streaming loads / stores of populations (variants selected at build time,
+// measured in tools/gpu_variants.sh): LBMR_LDVAR 0 = ld.global.nc, 1 = +
+// L2::256B prefetch, 2 = + L1::no_allocate + L2::256B, 3 = L1::no_allocate;
+// LBMR_STVAR 0 = st.global, 1 = st.global.cs (evict-first).
+#ifndef LBMR_LDVAR
+#define LBMR_LDVAR 1
+#endif
+#ifndef LBMR_STVAR
+#define LBMR_STVAR 0
+#endif
+template <typename T>
+__device__ __forceinline__ T ld_pop(const T* p) {
+#if LBMR_LDVAR == 0
+  return __ldg(p);
+#else
+  T v;
+  if constexpr (sizeof(T) == 4) {
+#if LBMR_LDVAR == 1
+    asm volatile("ld.global.nc.L2::256B.f32 %0, [%1];" : "=f"(v) : "l"(p));
+#elif LBMR_LDVAR == 2
+    asm volatile("ld.global.nc.L1::no_allocate.L2::256B.f32 %0, [%1];" : "=f"(v) : "l"(p));
+#else
+    asm volatile("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(v) : "l"(p));
+#endif
+  } else {
+#if LBMR_LDVAR == 1
+    asm volatile("ld.global.nc.L2::256B.f64 %0, [%1];" : "=d"(v) : "l"(p));
+#elif LBMR_LDVAR == 2
+    asm volatile("ld.global.nc.L1::no_allocate.L2::256B.f64 %0, [%1];" : "=d"(v) : "l"(p));
+#else
+    asm volatile("ld.global.nc.L1::no_allocate.f64 %0, [%1];" : "=d"(v) : "l"(p));
+#endif
+  }
+  return v;
+#endif
+}
+
+template <typename T>
+__device__ __forceinline__ void st_pop(T* p, T v) {
+#if LBMR_STVAR == 0
+  *p = v;
+#else
+  __stcs(p, v);
+#endif
+}
+
 // PRED = false: every link is a plain same-level pull.  PRED = true: load
 // only for fluid cells and existing neighbour blocks (links flagged slow are
 // loaded speculatively from the block arithmetic's source and overwritten by
@@ -303,8 +381,8 @@ __device__ __forceinline__ void pull_one(T (&g)[Q], const T* __restrict__ src, c
   const int nb = (q == 0) ? blk : __shfl_sync(FULL, rec, G.slot<q>());
   const unsigned off = (unsigned)nb * (unsigned)(Q * kCells) + (unsigned)G.local<q>();
   const T* p = src + q * kCells;  // constant part folds into the load's immediate offset
-  if (PRED) g[q] = (fluid && nb >= 0) ? __ldg(p + off) : T(0);
-  else g[q] = __ldg(p + off);
+  if (PRED) g[q] = (fluid && nb >= 0) ? ld_pop<T>(p + off) : T(0);
+  else g[q] = ld_pop<T>(p + off);
 }
 
 template <int Q, typename T, bool PRED, int... qs>
@@ -317,7 +395,7 @@ template <int Q, typename T>
 __device__ __forceinline__ void store_cell(const T (&g)[Q], T* __restrict__ dst, int blk, int t) {
   T* d = dst + (unsigned)blk * (unsigned)(Q * kCells) + t;
 #pragma unroll
-  for (int q = 0; q < Q; ++q) d[q * kCells] = g[q];
+  for (int q = 0; q < Q; ++q) st_pop<T>(d + q * kCells, g[q]);
 }
 
 // Minimum resident CTAs per SM (register budget 65536 / (256 * MINB)),
@@ -325,8 +403,18 @@ __device__ __forceinline__ void store_cell(const T (&g)[Q], T* __restrict__ dst,
 #ifndef LBMR_OCC_Q19F
 #define LBMR_OCC_Q19F 6
 #endif
-template <int Q, typename T>
-struct PlainOcc { static constexpr int value = (Q == 19 && sizeof(T) == 4) ? LBMR_OCC_Q19F : (sizeof(T) == 4 ? 3 : 2); };
+#ifndef LBMR_OCC_KBCF
+#define LBMR_OCC_KBCF 2
+#endif
+#ifndef LBMR_OCC_KBCD
+#define LBMR_OCC_KBCD 1
+#endif
+template <int Q, typename T, int COLL = LBM_BGK>
+struct PlainOcc {
+  static constexpr int value = COLL == LBM_KBC ? (sizeof(T) == 4 ? LBMR_OCC_KBCF : LBMR_OCC_KBCD)
+                               : (Q == 19 && sizeof(T) == 4) ? LBMR_OCC_Q19F
+                               : (sizeof(T) == 4 ? 3 : 2);
+};
 
 // ---------------------------------------------------------------- halo protocol
 // x-slab partition.  Blocks holding an owned cell of a cut
@@ -450,15 +538,23 @@ __device__ __forceinline__ void collide_cell(const StepParams<T>& P, int blk, in
   if (HALO) halo_store<Q, T>(P, g, blk, t);
 }
 
+// LBMR_CTA512: one CTA per 8^3 block (512 threads) instead of per half block
+#ifndef LBMR_CTA512
+#define LBMR_CTA512 0
+#endif
+constexpr int kStepThreads = LBMR_CTA512 ? 512 : 256;
+
 template <int Q, int COLL, typename T>
-__global__ void __launch_bounds__(256, PlainOcc<Q, T>::value) level_step_all(const StepParams<T> P) {
-  step_cell<Q, COLL, T, false>(P, blockIdx.x >> 1, ((blockIdx.x & 1) << 8) | threadIdx.x);
+__global__ void __launch_bounds__(kStepThreads, (PlainOcc<Q, T, COLL>::value * 256) / kStepThreads)
+    level_step_all(const StepParams<T> P) {
+  if (kStepThreads == 512) step_cell<Q, COLL, T, false>(P, blockIdx.x, threadIdx.x);
+  else step_cell<Q, COLL, T, false>(P, blockIdx.x >> 1, ((blockIdx.x & 1) << 8) | threadIdx.x);
 }
 
 // Partitioned variant: grid = 2 * max(nfluid, 1) CTAs; the first nbctas run
 // the halo protocol around their work.
 template <int Q, int COLL, typename T, bool STREAM>
-__global__ void __launch_bounds__(256, PlainOcc<Q, T>::value) level_step_halo(const StepParams<T> P) {
+__global__ void __launch_bounds__(256, PlainOcc<Q, T, COLL>::value) level_step_halo(const StepParams<T> P) {
   const int blk = blockIdx.x >> 1;
   const int t = ((blockIdx.x & 1) << 8) | threadIdx.x;
   const bool proto = (int)blockIdx.x < P.nbctas;
@@ -552,7 +648,7 @@ static void launch_typed(int kind, const void* params, cudaStream_t s) {
   if (p.nfluid <= 0) return;
   dim3 grid(2 * p.nfluid);
   if (kind == 1) level_collide<Q, COLL, T><<<grid, block, 0, s>>>(p);
-  else level_step_all<Q, COLL, T><<<grid, block, 0, s>>>(p);
+  else level_step_all<Q, COLL, T><<<dim3(p.nfluid * 512 / kStepThreads), dim3(kStepThreads), 0, s>>>(p);
 }
 
 // Load every kernel of the library now.  With lazy module loading (the CUDA
