@@ -239,6 +239,11 @@ __device__ __forceinline__ int opp_rt(int q) { return q == 0 ? 0 : ((q & 1) ? q 
 template <int Q, typename T>
 __device__ __forceinline__ void resolve_slow(const StepParams<T>& P, T (&g)[Q], uint32_t slow, unsigned j, int blk,
                                              int t) {
+  // values go to this thread's column of a shared buffer sv[q][threadIdx]
+  // (conflict-free for any q per lane) and are merged once at the end
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  T* sv = reinterpret_cast<T*>(smem_raw) + threadIdx.x;
+  const uint32_t all = slow;
   const unsigned own = (unsigned)blk * (unsigned)(Q * kCells) + (unsigned)t;
   while (slow) {
     int qb[4];
@@ -289,11 +294,12 @@ __device__ __forceinline__ void resolve_slow(const StepParams<T>& P, T (&g)[Q], 
         for (unsigned m = 0; m < n; ++m) acc += __ldg(P.fb + __ldg(c + m));
         val = acc / T(2 * n);
       }
-#pragma unroll
-      for (int qq = 0; qq < Q; ++qq)
-        if (qq == q) g[qq] = val;
+      sv[q * 256] = val;
     }
   }
+#pragma unroll
+  for (int q = 0; q < Q; ++q)
+    if (all & (1u << q)) g[q] = sv[q * 256];
 }
 
 // ---------------------------------------------------------------- fused kernel
@@ -635,20 +641,26 @@ __global__ void __launch_bounds__(512) macroscopic_kernel(const T* pop, const in
 }
 
 // ---------------------------------------------------------------- dispatch
+// dynamic shared memory of the stepping kernels: the slow-link staging
+// buffer sv[Q][256] of resolve_slow
+template <int Q, typename T>
+constexpr size_t slow_smem() { return (size_t)Q * 256 * sizeof(T); }
+
 template <int Q, int COLL, typename T>
 static void launch_typed(int kind, const void* params, cudaStream_t s) {
   const StepParams<T>& p = *static_cast<const StepParams<T>*>(params);
   dim3 block(256);
+  const size_t sm = slow_smem<Q, T>();
   if (p.nbctas > 0) {  // partitioned: always launched (the protocol must run)
     dim3 grid(2 * std::max(p.nfluid, 1));
     if (kind == 1) level_step_halo<Q, COLL, T, false><<<grid, block, 0, s>>>(p);
-    else level_step_halo<Q, COLL, T, true><<<grid, block, 0, s>>>(p);
+    else level_step_halo<Q, COLL, T, true><<<grid, block, sm, s>>>(p);
     return;
   }
   if (p.nfluid <= 0) return;
   dim3 grid(2 * p.nfluid);
   if (kind == 1) level_collide<Q, COLL, T><<<grid, block, 0, s>>>(p);
-  else level_step_all<Q, COLL, T><<<dim3(p.nfluid * 512 / kStepThreads), dim3(kStepThreads), 0, s>>>(p);
+  else level_step_all<Q, COLL, T><<<dim3(p.nfluid * 512 / kStepThreads), dim3(kStepThreads), sm, s>>>(p);
 }
 
 // Load every kernel of the library now.  With lazy module loading (the CUDA
@@ -657,6 +669,10 @@ static void launch_typed(int kind, const void* params, cudaStream_t s) {
 // a neighbour grid whose kernels this host thread has not launched yet.
 template <int Q, int COLL, typename T>
 static void preload_variant() {
+  cudaFuncSetAttribute(level_step_all<Q, COLL, T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                       (int)slow_smem<Q, T>());
+  cudaFuncSetAttribute(level_step_halo<Q, COLL, T, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                       (int)slow_smem<Q, T>());
   cudaFuncAttributes a;
   cudaFuncGetAttributes(&a, level_step_all<Q, COLL, T>);
   cudaFuncGetAttributes(&a, level_collide<Q, COLL, T>);
