@@ -245,11 +245,15 @@ __device__ __forceinline__ void resolve_slow(const StepParams<T>& P, T (&g)[Q], 
   T* sv = reinterpret_cast<T*>(smem_raw) + threadIdx.x;
   const uint32_t all = slow;
   const unsigned own = (unsigned)blk * (unsigned)(Q * kCells) + (unsigned)t;
+#ifndef LBMR_SLOW_NB
+#define LBMR_SLOW_NB 4
+#endif
+  constexpr int NB = (Q == 19 && sizeof(T) == 4) ? 4 : LBMR_SLOW_NB;
   while (slow) {
-    int qb[4];
-    uint2 eb[4];
+    int qb[NB];
+    uint2 eb[NB];
 #pragma unroll
-    for (int b = 0; b < 4; ++b) {
+    for (int b = 0; b < NB; ++b) {
       qb[b] = -1;
       eb[b] = make_uint2(0u, 0u);
       if (slow) {
@@ -259,9 +263,9 @@ __device__ __forceinline__ void resolve_slow(const StepParams<T>& P, T (&g)[Q], 
         ++j;
       }
     }
-    T v[4];
+    T v[NB];
 #pragma unroll
-    for (int b = 0; b < 4; ++b) {
+    for (int b = 0; b < NB; ++b) {
       v[b] = T(0);
       if (qb[b] >= 0) {
         const unsigned tag = eb[b].y >> 28;
@@ -271,7 +275,7 @@ __device__ __forceinline__ void resolve_slow(const StepParams<T>& P, T (&g)[Q], 
       }
     }
 #pragma unroll
-    for (int b = 0; b < 4; ++b) {
+    for (int b = 0; b < NB; ++b) {
       const int q = qb[b];
       if (q < 0) continue;
       const unsigned tag = eb[b].y >> 28;
