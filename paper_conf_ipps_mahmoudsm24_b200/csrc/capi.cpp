@@ -57,6 +57,7 @@ struct DevLevel {
   uint32_t* links = nullptr;
   uint32_t* coal = nullptr;
   int32_t* bpeer = nullptr;
+  uint32_t* ghost_fill = nullptr;
   void* pop[2] = {nullptr, nullptr};
   // neighbour rank on each side: its population buffers and the halo cell
   // index (in its grid) of every entry of our send list
@@ -187,7 +188,10 @@ StepParams<T> make_params(const lbm_grid* g, int L, int64_t k) {
   p.omega = (T)g->omega[L];
   for (int a = 0; a < 3; ++a) p.periodic[a] = g->desc.periodic[a];
   p.face_cls = g->face_dev;
-  p.nfluid = g->n_ranks > 1 ? g->host[L].nlaunch : g->host[L].nfluid;
+  p.nfluid = g->host[L].nlaunch;
+  p.ghost_fill = D.ghost_fill;
+  p.nghost = (int32_t)(g->host[L].ghost_fill.size() / 2);
+  if (L > 0) p.gsrc = static_cast<const T*>(g->dev[L - 1].pop[((k + 2) / 2) & 1]);  // C_{L-1}^{ceil((k+1)/2)}
   if (g->n_ranks > 1) {
     const HostLevel& H = g->host[L];
     p.nbctas = std::max(2 * H.nboundary, 1);
@@ -541,6 +545,7 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     if ((s = dev_upload(g, &D.links, H.links))) return cleanup(s);
     if ((s = dev_upload(g, &D.coal, H.coal))) return cleanup(s);
     if ((s = dev_upload(g, &D.bpeer, H.bpeer))) return cleanup(s);
+    if ((s = dev_upload(g, &D.ghost_fill, H.ghost_fill))) return cleanup(s);
     for (int b = 0; b < 2; ++b) {
       if ((s = dev_alloc(g, &D.pop[b], pop_bytes(g, L)))) return cleanup(s);
       if (cudaMemset(D.pop[b], 0, pop_bytes(g, L)) != cudaSuccess) return cleanup(fail(LBM_E_CUDA, "memset"));
@@ -551,6 +556,7 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     std::vector<uint32_t>().swap(H.links);
     std::vector<uint32_t>().swap(H.coal);
     std::vector<int32_t>().swap(H.nbr);
+    std::vector<uint8_t>().swap(H.ghost);
   }
   void* p;
   if (g->n_ranks > 1) {  // halo-protocol flags, own allocation so it can be shared by CUDA IPC

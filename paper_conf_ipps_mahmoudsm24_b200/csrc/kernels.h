@@ -43,6 +43,11 @@ struct StepParams {
   int32_t periodic[3];
   const uint8_t* face_cls;      // [27] BC class of an out-of-domain source, by outside pattern
   int32_t nfluid;               // blocks launched (owned fluid blocks, cut-plane blocks first)
+  // explosion ghosts of the destination buffer, refreshed from the coarse
+  // post-collision state the NEXT kernel of this level reads (Eq.10)
+  const uint32_t* ghost_fill;   // pairs {ghost cell, parent cell}
+  int32_t nghost;
+  const T* gsrc;                // C_{L-1}^{ceil((k+1)/2)}
   // ---- x-slab partition (multi-GPU); unused when nbctas == 0 -------------
   int32_t nbctas;               // CTAs taking part in the halo protocol (cut-plane blocks, >= 1)
   int32_t nboundary;            // cut-plane blocks (stored and launched first)

@@ -408,6 +408,21 @@ __device__ __forceinline__ void store_cell(const T (&g)[Q], T* __restrict__ dst,
   for (int q = 0; q < Q; ++q) st_pop<T>(d + q * kCells, g[q]);
 }
 
+// Explosion ghosts: ghost cell g of level L holds its parent's
+// C_{L-1} populations, so interface cells pull the exploded value (Eq.10)
+// as a plain same-level load.  One thread per ghost, all Q planes.
+template <int Q, typename T>
+__device__ __forceinline__ void ghost_fill_one(const StepParams<T>& P, int i) {
+  if (i >= P.nghost) return;
+  const uint32_t gc = __ldg(P.ghost_fill + 2 * i), pc = __ldg(P.ghost_fill + 2 * i + 1);
+  T* d = P.dst + (gc >> 9) * (unsigned)(Q * kCells) + (gc & 511u);
+  const T* s = P.gsrc + (pc >> 9) * (unsigned)(Q * kCells) + (pc & 511u);
+#pragma unroll
+  for (int q = 0; q < Q; ++q) d[q * kCells] = __ldg(s + q * kCells);
+}
+
+__host__ __device__ constexpr int ghost_ctas(int n) { return (n + 255) / 256; }
+
 // Minimum resident CTAs per SM (register budget 65536 / (256 * MINB)),
 // chosen per variant from ptxas -v and measurement.
 #ifndef LBMR_OCC_Q19F
@@ -443,33 +458,11 @@ __device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long
 }
 
 template <typename T>
-__device__ __forceinline__ void halo_wait(const StepParams<T>& P) {
-  if (threadIdx.x == 0) {
-    const unsigned long long mine = *(volatile unsigned long long*)(P.flags + 2);
-    for (int s = 0; s < 2; ++s)
-      if (P.has_nb[s]) {
-#ifdef LBMR_DEBUG_HALO
-        long long spins = 0;
-#endif
-        while (ld_acquire_sys(P.flags + s) < mine) {
-          __nanosleep(256);
-#ifdef LBMR_DEBUG_HALO
-          if (++spins == 2000000)
-            printf("halo_wait stuck: cta %d side %d flag %llu mine %llu nfluid %d nbctas %d\n", blockIdx.x, s,
-                   ld_acquire_sys(P.flags + s), mine, P.nfluid, P.nbctas);
-#endif
-        }
-      }
-  }
-  __syncthreads();
-}
-
-template <typename T>
-__device__ __forceinline__ void halo_signal(const StepParams<T>& P) {
+__device__ __forceinline__ void halo_signal(const StepParams<T>& P, int nproto) {
   __threadfence_system();
   __syncthreads();
   if (threadIdx.x == 0) {
-    if (atomicAdd(P.flags + 3, 1ull) == (unsigned long long)(P.nbctas - 1)) {
+    if (atomicAdd(P.flags + 3, 1ull) == (unsigned long long)(nproto - 1)) {
       P.flags[3] = 0ull;
       P.flags[2] += 1ull;
       __threadfence_system();
@@ -557,27 +550,54 @@ constexpr int kStepThreads = LBMR_CTA512 ? 512 : 256;
 template <int Q, int COLL, typename T>
 __global__ void __launch_bounds__(kStepThreads, (PlainOcc<Q, T, COLL>::value * 256) / kStepThreads)
     level_step_all(const StepParams<T> P) {
+  const int main = P.nfluid * 512 / kStepThreads;
+  if ((int)blockIdx.x >= main) {  // trailing CTAs refresh the explosion ghosts
+    ghost_fill_one<Q, T>(P, ((int)blockIdx.x - main) * kStepThreads + threadIdx.x);
+    return;
+  }
   if (kStepThreads == 512) step_cell<Q, COLL, T, false>(P, blockIdx.x, threadIdx.x);
   else step_cell<Q, COLL, T, false>(P, blockIdx.x >> 1, ((blockIdx.x & 1) << 8) | threadIdx.x);
 }
 
 // Partitioned variant: grid = 2 * max(nfluid, 1) CTAs; the first nbctas run
 // the halo protocol around their work.
+// One thread waits until every neighbour has completed the cut-plane part of
+// all kernels this rank has completed (its bumps of our flag reach our
+// kernel count).  A separate one-CTA launch, so that no CTA of a level kernel
+// ever spins: partitions emulated on one device cannot starve each other.
+__global__ void halo_wait_kernel(const unsigned long long* flags, int nb0, int nb1) {
+  const unsigned long long mine = *(volatile const unsigned long long*)(flags + 2);
+  if (nb0)
+    while (ld_acquire_sys(flags + 0) < mine) __nanosleep(256);
+  if (nb1)
+    while (ld_acquire_sys(flags + 1) < mine) __nanosleep(256);
+}
+
 template <int Q, int COLL, typename T, bool STREAM>
 __global__ void __launch_bounds__(256, PlainOcc<Q, T, COLL>::value) level_step_halo(const StepParams<T> P) {
   const int blk = blockIdx.x >> 1;
   const int t = ((blockIdx.x & 1) << 8) | threadIdx.x;
-  const bool proto = (int)blockIdx.x < P.nbctas;
-  if (proto) halo_wait<T>(P);
-  if (blk < P.nfluid) {
+  const int main = 2 * max(P.nfluid, 1);
+  // the wait happened in halo_wait_kernel just before this launch; cut-plane
+  // CTAs (which write the neighbour's halo) and ghost-refresh CTAs (which may
+  // read L-1 halo cells) count towards this kernel's completion signal
+  const bool fill = (int)blockIdx.x >= main;
+  const bool proto = (int)blockIdx.x < P.nbctas || fill;
+  if (fill) {
+    ghost_fill_one<Q, T>(P, ((int)blockIdx.x - main) * 256 + threadIdx.x);
+  } else if (blk < P.nfluid) {
     if (STREAM) step_cell<Q, COLL, T, true>(P, blk, t);
     else collide_cell<Q, COLL, T, true>(P, blk, t);
   }
-  if (proto) halo_signal<T>(P);
+  if (proto) halo_signal<T>(P, P.nbctas + ghost_ctas(P.nghost));
 }
 
 template <int Q, int COLL, typename T>
 __global__ void __launch_bounds__(256) level_collide(const StepParams<T> P) {
+  if ((int)blockIdx.x >= 2 * P.nfluid) {
+    ghost_fill_one<Q, T>(P, ((int)blockIdx.x - 2 * P.nfluid) * 256 + threadIdx.x);
+    return;
+  }
   collide_cell<Q, COLL, T, false>(P, blockIdx.x >> 1, ((blockIdx.x & 1) << 8) | threadIdx.x);
 }
 
@@ -655,16 +675,21 @@ static void launch_typed(int kind, const void* params, cudaStream_t s) {
   const StepParams<T>& p = *static_cast<const StepParams<T>*>(params);
   dim3 block(256);
   const size_t sm = slow_smem<Q, T>();
+  const int gc = ghost_ctas(p.nghost);
   if (p.nbctas > 0) {  // partitioned: always launched (the protocol must run)
-    dim3 grid(2 * std::max(p.nfluid, 1));
+    halo_wait_kernel<<<1, 1, 0, s>>>(p.flags, p.has_nb[0], p.has_nb[1]);
+    dim3 grid(2 * std::max(p.nfluid, 1) + gc);
     if (kind == 1) level_step_halo<Q, COLL, T, false><<<grid, block, 0, s>>>(p);
     else level_step_halo<Q, COLL, T, true><<<grid, block, sm, s>>>(p);
     return;
   }
-  if (p.nfluid <= 0) return;
-  dim3 grid(2 * p.nfluid);
-  if (kind == 1) level_collide<Q, COLL, T><<<grid, block, 0, s>>>(p);
-  else level_step_all<Q, COLL, T><<<dim3(p.nfluid * 512 / kStepThreads), dim3(kStepThreads), sm, s>>>(p);
+  if (p.nfluid <= 0 && p.nghost <= 0) return;
+  if (kind == 1) {
+    level_collide<Q, COLL, T><<<dim3(2 * p.nfluid + gc), block, 0, s>>>(p);
+  } else {
+    const int gct = (p.nghost + kStepThreads - 1) / kStepThreads;
+    level_step_all<Q, COLL, T><<<dim3(p.nfluid * 512 / kStepThreads + gct), dim3(kStepThreads), sm, s>>>(p);
+  }
 }
 
 // Load every kernel of the library now.  With lazy module loading (the CUDA
@@ -692,6 +717,7 @@ void preload_kernels() {
   preload_variant<27, LBM_BGK, double>();
   preload_variant<27, LBM_KBC, double>();
   cudaFuncAttributes a;
+  cudaFuncGetAttributes(&a, halo_wait_kernel);
   cudaFuncGetAttributes(&a, init_eq_kernel<19, float>);
   cudaFuncGetAttributes(&a, init_eq_kernel<27, float>);
   cudaFuncGetAttributes(&a, init_eq_kernel<19, double>);

@@ -165,15 +165,18 @@ def test_rejects_bad_arguments():
 
 
 def test_builder_statistics_of_the_baseline_configs():
-    """Interface structure of cfg3/cfg5: share of fluid
-    leaves with a non-same-level/BC link and of blocks holding one."""
+    """Interface structure of cfg3/cfg5.  Level 0 has no
+    coarser neighbour, so its share of leaves with a non-plain link is the
+    survey's interface share (6.4 % / 9.0 %); on finer levels the explosion
+    links are plain pulls from ghost cells, so only coalescence / BC / wall
+    cells remain on the slow path there (well below the survey's 3-7 %)."""
     gi = lbmr.analyze_problem(I.sphere3())
     assert list(gi.leaves[:3]) == [3375104, 5373952, 9299808]
     sc = [gi.special_cells[L] / gi.leaves[L] for L in range(3)]
-    sb = [gi.special_blocks[L] / gi.blocks[L] for L in range(3)]
-    assert [round(v, 3) for v in sc] == [0.064, 0.052, 0.031]
-    assert [round(v, 2) for v in sb] == [0.50, 0.41, 0.23]
+    assert round(sc[0], 3) == 0.064
+    assert sc[1] < 0.052 and sc[2] < 0.031 * 0.2
     gi = lbmr.analyze_problem(I.tunnel4())
     assert list(gi.leaves[:4]) == [1413300, 4670400, 8940544, 33155968]
     assert gi.kernels_per_step == 15
-    assert abs(gi.special_cells[3] / gi.leaves[3] - 0.029) < 0.002
+    assert round(gi.special_cells[0] / gi.leaves[0], 3) == 0.090
+    assert gi.special_cells[3] / gi.leaves[3] < 0.01
