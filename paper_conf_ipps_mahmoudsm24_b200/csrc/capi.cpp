@@ -58,6 +58,8 @@ struct DevLevel {
   uint32_t* coal = nullptr;
   int32_t* bpeer = nullptr;
   uint32_t* ghost_fill = nullptr;
+  uint32_t* coal_fill = nullptr;
+  uint32_t* coal_cand = nullptr;
   void* pop[2] = {nullptr, nullptr};
   // neighbour rank on each side: its population buffers and the halo cell
   // index (in its grid) of every entry of our send list
@@ -215,6 +217,17 @@ void launch_F_typed(lbm_grid* g, int L, int64_t k, int kind) {
   if (kind == 1) {  // prologue collision
     launch_level_step(g->Q, g->coll, g->prec, 1, &p, g->stream);
     return;
+  }
+  // coalescence ghosts of C_L^k from C_{L+1}^{2k-1} and C_{L+1}^{2k} (both ready now)
+  const HostLevel& H = g->host[L];
+  if (L + 1 < g->levels && !H.coal_fill.empty()) {
+    if (g->n_ranks > 1) {
+      // the gather reads L+1 halo cells: it follows the neighbour wait of F_L^k,
+      // which launch_level_step issues first; issue an explicit wait here instead
+      launch_halo_wait(p.flags, p.has_nb[0], p.has_nb[1], g->stream);
+    }
+    launch_coalesce(g->Q, g->prec, g->dev[L + 1].pop[1], g->dev[L + 1].pop[0], g->dev[L].pop[k & 1],
+                    g->dev[L].coal_fill, g->dev[L].coal_cand, (int32_t)(H.coal_fill.size() / 2), g->stream);
   }
   launch_level_step(g->Q, g->coll, g->prec, 0, &p, g->stream);
 }
@@ -546,6 +559,8 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     if ((s = dev_upload(g, &D.coal, H.coal))) return cleanup(s);
     if ((s = dev_upload(g, &D.bpeer, H.bpeer))) return cleanup(s);
     if ((s = dev_upload(g, &D.ghost_fill, H.ghost_fill))) return cleanup(s);
+    if ((s = dev_upload(g, &D.coal_fill, H.coal_fill))) return cleanup(s);
+    if ((s = dev_upload(g, &D.coal_cand, H.coal_cand))) return cleanup(s);
     for (int b = 0; b < 2; ++b) {
       if ((s = dev_alloc(g, &D.pop[b], pop_bytes(g, L)))) return cleanup(s);
       if (cudaMemset(D.pop[b], 0, pop_bytes(g, L)) != cudaSuccess) return cleanup(fail(LBM_E_CUDA, "memset"));

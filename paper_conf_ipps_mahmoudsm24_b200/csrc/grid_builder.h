@@ -36,8 +36,10 @@ struct HostLevel {
   std::vector<int32_t> bpeer;         // [nboundary][2][512] index into send[side] or -1
   // explosion ghosts (ABSENT cells pulled by fluid leaves, parent a fluid
   // leaf at L-1): stored, refreshed by the level's previous kernel
-  std::vector<uint8_t> ghost;         // [nblocks*512] host-only flag
+  std::vector<uint8_t> ghost;         // [nblocks*512] host only: 1 explosion ghost, 2 coalescence ghost
   std::vector<uint32_t> ghost_fill;   // pairs {ghost cell at L, parent cell at L-1} (block*512+local)
+  std::vector<uint32_t> coal_fill;    // pairs {dest population index (ghost, q), (|B|-1) << 26 | first candidate}
+  std::vector<uint32_t> coal_cand;    // fine candidate population indices (level L+1)
   std::vector<int32_t> plain_ids;     // fluid blocks without special cells (Morton order)
   std::vector<int32_t> special_ids;   // the others (Morton order)
 };

@@ -59,6 +59,17 @@ struct StepParams {
   const int32_t* bpeer;         // [nboundary][2][512] send-list index of a cut-plane cell, or -1
 };
 
+// Coalescence gather (Eq.11) into the coarse ghosts of `dst` (= C_L^k's
+// buffer, read next by F_L^k): for entry i, dst[fill[2i]] = (sum_B fa + sum_B fb)
+// / (2|B|) over the candidates cand[(fill[2i+1] & 0x3ffffff) ...], |B| =
+// (fill[2i+1] >> 26) + 1.
+void launch_coalesce(int Q, int precision, const void* fa, const void* fb, void* dst, const uint32_t* fill,
+                     const uint32_t* cand, int32_t n, cudaStream_t s);
+
+// One-thread kernel: wait until both neighbours (has_nb) have completed the
+// cut-plane part of every kernel this rank has completed.
+void launch_halo_wait(const unsigned long long* flags, int nb0, int nb1, cudaStream_t s);
+
 // Force-load every kernel (see level_step.cu).
 void preload_kernels();
 

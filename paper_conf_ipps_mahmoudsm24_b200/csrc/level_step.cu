@@ -664,6 +664,39 @@ __global__ void __launch_bounds__(512) macroscopic_kernel(const T* pop, const in
   }
 }
 
+// Coalescence ghosts: one thread per (ghost cell, q) entry.
+// Fine candidates summed in candidate order, first substep then second, like
+// the oracle (Eq.11, n = 2|B|, R-A2/R-A3).
+template <typename T>
+__global__ void __launch_bounds__(256) coalesce_kernel(const T* __restrict__ fa, const T* __restrict__ fb,
+                                                       T* __restrict__ dst, const uint32_t* __restrict__ fill,
+                                                       const uint32_t* __restrict__ cand, int n) {
+  const int i = blockIdx.x * 256 + threadIdx.x;
+  if (i >= n) return;
+  const uint32_t d = __ldg(fill + 2 * i), w = __ldg(fill + 2 * i + 1);
+  const unsigned cnt = (w >> 26) + 1u;
+  const uint32_t* c = cand + (w & 0x3ffffffu);
+  T acc = T(0);
+  for (unsigned m = 0; m < cnt; ++m) acc += __ldg(fa + __ldg(c + m));
+  for (unsigned m = 0; m < cnt; ++m) acc += __ldg(fb + __ldg(c + m));
+  dst[d] = acc / T(2 * cnt);
+}
+
+void launch_halo_wait(const unsigned long long* flags, int nb0, int nb1, cudaStream_t s) {
+  halo_wait_kernel<<<1, 1, 0, s>>>(flags, nb0, nb1);
+}
+
+void launch_coalesce(int Q, int precision, const void* fa, const void* fb, void* dst, const uint32_t* fill,
+                     const uint32_t* cand, int32_t n, cudaStream_t s) {
+  (void)Q;
+  if (n <= 0) return;
+  const int grid = (n + 255) / 256;
+  if (precision == LBM_FP32)
+    coalesce_kernel<float><<<grid, 256, 0, s>>>((const float*)fa, (const float*)fb, (float*)dst, fill, cand, n);
+  else
+    coalesce_kernel<double><<<grid, 256, 0, s>>>((const double*)fa, (const double*)fb, (double*)dst, fill, cand, n);
+}
+
 // ---------------------------------------------------------------- dispatch
 // dynamic shared memory of the stepping kernels: the slow-link staging
 // buffer sv[Q][256] of resolve_slow
@@ -718,6 +751,8 @@ void preload_kernels() {
   preload_variant<27, LBM_KBC, double>();
   cudaFuncAttributes a;
   cudaFuncGetAttributes(&a, halo_wait_kernel);
+  cudaFuncGetAttributes(&a, coalesce_kernel<float>);
+  cudaFuncGetAttributes(&a, coalesce_kernel<double>);
   cudaFuncGetAttributes(&a, init_eq_kernel<19, float>);
   cudaFuncGetAttributes(&a, init_eq_kernel<27, float>);
   cudaFuncGetAttributes(&a, init_eq_kernel<19, double>);
