@@ -41,6 +41,15 @@ CONFIGS = {
     "uniform512": (lambda: I.uniform(512), "cfg2 uniform512: D3Q19 BGK, single level 512^3 periodic"),
     "cavity2": (lambda: I.cavity2(), "cfg1 cavity2: D3Q19 BGK, 2 levels, 32^3 coarse"),
 }
+# the paper's Tab. I sphere sweep (D3Q27 KBC, 3 levels, fp64 like the paper)
+for _s in (1, 2, 3):
+    CONFIGS[f"sphere_tab1_s{_s}"] = (
+        (lambda s=_s: I.sphere_tab1(s)),
+        f"Tab. I sphere row {_s}: D3Q27 KBC, 3 levels, {272 * _s}x{192 * _s}x{272 * _s} finest-equivalent, Re=4000")
+DEFAULT_PRECISION = {f"sphere_tab1_s{_s}": "fp64" for _s in (1, 2, 3)}
+# the paper's own number for exactly this metric and workload (A100, fp64), Tab. I
+PAPER_MLUPS = {f"sphere_tab1_s{_s}": I.TAB1[_s]["ours_mlups"] for _s in (1, 2, 3)}
+SCHEDULES = {"fused": 0, "unfused": 1, "nograph": 2, "unfused_nograph": 3}
 # bounded oracle sample for --impl reference (one coarse step per timed step)
 REF_SAMPLE = {
     "tunnel4": (lambda: I.tunnel4(scale=5), "tunnel4 geometry at 1/5 scale (40x21x21 coarse, 4 levels)"),
@@ -50,6 +59,8 @@ REF_SAMPLE = {
     "uniform512": (lambda: I.uniform(64), "uniform periodic 64^3"),
     "cavity2": (lambda: I.cavity2(), "cavity2 (full size)"),
 }
+for _s in (1, 2, 3):
+    REF_SAMPLE[f"sphere_tab1_s{_s}"] = (lambda: I.sphere_tab1(1), "Tab. I sphere row 1 (272x192x272 finest-equivalent)")
 
 
 def updates_per_step(leaves):
@@ -168,11 +179,16 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="tunnel4", choices=sorted(CONFIGS))
-    ap.add_argument("--precision", default="fp32", choices=["fp32", "fp64"])
+    ap.add_argument("--precision", default=None, choices=["fp32", "fp64"],
+                    help="default fp32 (fp64 for the Tab. I sphere configs, the paper's precision)")
+    ap.add_argument("--schedule", default="fused", choices=sorted(SCHEDULES),
+                    help="fusion ablation (lbm_set_schedule); the default is the product schedule")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--profile-steps", type=int, default=10)
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
+    if args.precision is None:
+        args.precision = DEFAULT_PRECISION.get(args.config, "fp32")
     ws, rank, local = dist_setup()
 
     if args.impl == "reference":
@@ -209,6 +225,7 @@ def main():
             if lbmr.g_has(g, side):
                 g.halo_connect(side, allb[(rank + (1 if side else -1)) % ws][1 - side])
     lbmr.init_from_problem(g, prob)
+    g.set_schedule(SCHEDULES[args.schedule])
     setup_s = time.perf_counter() - t0
     info = g.info()
     leaves_local = [int(info.leaves[L]) for L in range(prob.levels)]
@@ -218,7 +235,9 @@ def main():
         torch.distributed.all_reduce(t)
         leaves = [int(v) for v in t.tolist()]
     upd = updates_per_step(leaves)
-    kernels_per_step = int(info.kernels_per_step)
+    launches_per_step = int(info.launches_per_step)
+    if SCHEDULES[args.schedule] & 1:  # unfused: stream + collide kernel per level-substep
+        launches_per_step += int(info.kernels_per_step)
 
     g.step(args.warmup)
     g.synchronize()
@@ -305,12 +324,14 @@ def main():
         line = {
             "metric": METRIC, "value": value, "unit": "MLUPS", "n_gpus": ws, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
-            "scaling": "strong", "vs_baseline": None,
+            "scaling": "strong",
+            "vs_baseline": (value / PAPER_MLUPS[args.config]) if args.config in PAPER_MLUPS and ws == 1 else None,
             "dtype": "f32" if prec == lbmr.FP32 else "f64", "data": "synthetic",
             "config": {"workload": desc, "levels": prob.levels, "leaves": leaves, "updates_per_step": upd,
                        "parallelism": f"x-slabs x{ws} (halo peer stores over NVLink)" if ws > 1 else "single",
                        "l2": f"working set {dev_bytes / 1e9:.2f} GB > 126 MB L2 (no flush needed)",
-                       "precision": args.precision, "setup_s": round(setup_s, 2)},
+                       "precision": args.precision, "schedule": args.schedule, "setup_s": round(setup_s, 2),
+                       **({"paper_a100_fp64_mlups": PAPER_MLUPS[args.config]} if args.config in PAPER_MLUPS else {})},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "kernel": f"level_step L{dom}",
                          "bytes_per_update": bpu, "peak_source": peak_src,
@@ -319,7 +340,7 @@ def main():
             "per_level": per_level,
             "cpu_baseline": cpu,
             "e2e": e2e,
-            "gpu_launches": kernels_per_step * args.steps,
+            "gpu_launches": launches_per_step * args.steps,
             "clocks": clocks,
         }
         print(json.dumps(line), flush=True)

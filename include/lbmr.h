@@ -85,6 +85,9 @@ typedef struct {
   int64_t total_blocks[16];          /* all stored blocks incl. refined/BC-only                   */
   int64_t device_bytes;              /* device memory held by the grid                            */
   int64_t steps_done;                /* coarse steps since the last init                          */
+  int64_t launches_per_step;         /* every kernel of one fused coarse step: the level steps plus
+                                        one coalescence gather before each F_L^k whose level has
+                                        coalescence ghosts                                          */
 } lbm_grid_info;
 
 /* Build the block-sparse multi-level grid (§V) from per-level masks.
@@ -136,6 +139,39 @@ lbm_status lbm_grid_get_info(const lbm_grid* g, lbm_grid_info* info);
  * NULL).  Synchronises. */
 lbm_status lbm_profile_levels(lbm_grid* g, int32_t n_coarse, double* ms_per_level,
                               int64_t* launches_per_level);
+
+/* Kernel schedule of lbm_step / lbm_profile_levels (bit flags; default 0).
+ *  LBM_SCHED_FUSED     one fused kernel F_L^k per level-substep (stream +
+ *                      Explosion + Coalescence + BC + collide), 2Q values
+ *                      moved per leaf — the paper's fully fused design
+ *                      (Fig. 4f) in the pipelined order.
+ *  LBM_SCHED_UNFUSED   ablation (Fig. 9): per level-substep a
+ *                      stream-only kernel S_L^k then an in-place collision
+ *                      C_L^{k+1} (4Q values per leaf).  Bitwise identical
+ *                      results.  Single rank only (LBM_E_UNSUPPORTED).
+ *  LBM_SCHED_NO_GRAPH  launch the kernels one by one instead of replaying
+ *                      the captured CUDA graph (launch-overhead ablation).
+ * Takes effect at the next lbm_step; synchronises the grid's stream. */
+enum { LBM_SCHED_FUSED = 0, LBM_SCHED_UNFUSED = 1, LBM_SCHED_NO_GRAPH = 2 };
+lbm_status lbm_set_schedule(lbm_grid* g, int32_t mode);
+
+/* Checkpoint / resume.  The state at a coarse-step
+ * boundary is, per level, the current population buffer (post-collision
+ * C_L^{k+1} with its explosion/coalescence ghosts, or the initial
+ * post-streaming state before the first step) plus the step counter.
+ *  lbm_checkpoint_size:  bytes a checkpoint of this grid takes (header +
+ *                        sum_L blocks_L * Q * 512 * sizeof(precision)).
+ *  lbm_checkpoint_save:  synchronises, copies the state into the caller's
+ *                        host buffer `host` of `capacity` bytes
+ *                        (LBM_E_INVAL if too small).
+ *  lbm_checkpoint_load:  restores a checkpoint into a grid created from the
+ *                        SAME desc/masks (same rank of the same partition);
+ *                        LBM_E_INVAL if it belongs to another layout.  The
+ *                        continued run is bitwise identical to an
+ *                        uninterrupted one.  The caller owns `host`. */
+lbm_status lbm_checkpoint_size(const lbm_grid* g, int64_t* bytes);
+lbm_status lbm_checkpoint_save(lbm_grid* g, void* host, int64_t capacity);
+lbm_status lbm_checkpoint_load(lbm_grid* g, const void* host, int64_t size);
 
 /* Block until all work enqueued on the grid's stream is done. */
 lbm_status lbm_synchronize(lbm_grid* g);

@@ -291,12 +291,66 @@ def tunnel4(scale: int = 1) -> Problem:
     )
 
 
+def sphere_tab1(size: int = 1, re: float = 4000.0, collision: str = "kbc", Q: int = 27) -> Problem:
+    """the paper's Tab. I flow over a sphere (P:L292-300,
+    Fig. 8): D3Q27 KBC, 3 levels, virtual wind tunnel of (272, 192, 272) * size
+    finest cells (size = 1, 2, 3 are the three rows of Tab. I), i.e. a coarse
+    grid of (68, 48, 68) * size.  The paper prints the leaf distribution only
+    (finest, middle, coarse = 0.602, 0.296, 0.175 M at size 1, x size^3), not the
+    refinement regions; this recipe uses two nested boxes
+    (coarse units, x size):  L1 x[4,48) y[8,40) z[17,50);  L2 x[13,40) y[14,33)
+    z[24,43), giving 0.607 / 0.294 / 0.175 M leaves at size 1 (+0.8 / -0.8 /
+    +0.3 %).  Sphere of radius R = 16 * size finest cells centred at
+    (80, 94, 134) * size finest units (cells whose centre is inside are
+    no-slip BC leaves).  -x velocity inlet (0.05, 0, 0), +x outflow, +-y, +-z
+    no-slip.  Re = u_in R / nu_finest = 4000 (Fig. 8 caption) =>
+    nu_0 = nu_2 / 4, omega0 = 1 / (3 nu_0 + 1/2) (Eq.4)."""
+    s = int(size)
+    if s < 1:
+        raise ValueError("size >= 1")
+    n = (68 * s, 48 * s, 68 * s)
+    b1 = ((4 * s, 48 * s), (8 * s, 40 * s), (17 * s, 50 * s))
+    b2 = ((13 * s, 40 * s), (14 * s, 33 * s), (24 * s, 43 * s))
+    masks = _box_masks(n, [b1, b2])
+    f = masks[2]
+    R = 16.0 * s
+    cx, cy, cz = 80.0 * s, 94.0 * s, 134.0 * s
+    (x0, x1), (y0, y1), (z0, z1) = [(a * 4, b * 4) for a, b in b2]
+    xs = np.arange(x0, x1) + 0.5 - cx
+    ys = np.arange(y0, y1) + 0.5 - cy
+    zs = np.arange(z0, z1) + 0.5 - cz
+    inside = (xs[:, None, None] ** 2 + ys[None, :, None] ** 2 + zs[None, None, :] ** 2) < R * R
+    f[x0:x1, y0:y1, z0:z1][inside] = CLS_WALL
+    nu2 = 0.05 * R / re
+    nu0 = nu2 / 4.0
+    return Problem(
+        name=f"sphere_tab1_s{s}" + ("" if (collision, Q) == ("kbc", 27) else f"_{collision}{Q}"),
+        nx=n[0], ny=n[1], nz=n[2], masks=masks,
+        face_bc=(CLS_LID, CLS_OUT, CLS_WALL, CLS_WALL, CLS_WALL, CLS_WALL),
+        Q=Q, collision=collision, omega0=1.0 / (3 * nu0 + 0.5),
+        bc={CLS_WALL: (BC_NOSLIP, (0.0, 0.0, 0.0)), CLS_LID: (BC_VELOCITY, (0.05, 0.0, 0.0)),
+            CLS_OUT: (BC_OUTFLOW, (0.0, 0.0, 0.0))},
+        uniform_u=(0.05, 0.0, 0.0),
+    )
+
+
+# Tab. I (P:L296-298): leaves (finest, middle, coarse) in millions and the
+# paper's A100 fp64 MLUPS of its modified baseline (Fig. 4b) and optimised
+# (Fig. 4f) implementations — context for bench.py's vs_baseline.
+TAB1 = {
+    1: dict(leaves_M=(0.602, 0.296, 0.175), baseline_mlups=482.63, ours_mlups=1081.67),
+    2: dict(leaves_M=(4.81, 2.37, 1.40), baseline_mlups=1115.80, ours_mlups=1646.37),
+    3: dict(leaves_M=(16.25, 8.0, 4.74), baseline_mlups=1299.7, ours_mlups=1805.03),
+}
+
+
 CONFIGS = {
     "cavity2": cavity2,
     "uniform512": uniform,
     "sphere3": sphere3,
     "cavity4_kbc": cavity4_kbc,
     "tunnel4": tunnel4,
+    "sphere_tab1": sphere_tab1,
 }
 
 

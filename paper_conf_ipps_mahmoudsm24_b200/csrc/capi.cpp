@@ -89,6 +89,7 @@ struct lbm_grid {
   bool needs_prologue = true;
   bool init_locked = false;  // a step ran since the last init_uniform
   bool broken = false;
+  int sched = LBM_SCHED_FUSED;  // lbm_set_schedule
   int64_t steps = 0;
   int64_t device_bytes = 0;
   std::vector<void*> allocs;
@@ -175,7 +176,7 @@ StepParams<T> make_params(const lbm_grid* g, int L, int64_t k) {
   p.fine = view_of(g, L + 1);
   p.nbr = D.nbr;
   p.special_slot = D.special_slot;
-  p.cellinfo = reinterpret_cast<const uint2*>(D.cellinfo);
+  p.cellinfo = reinterpret_cast<const uint4*>(D.cellinfo);
   p.links = reinterpret_cast<const uint2*>(D.links);
   p.coal = D.coal;
   p.origin = D.origin;
@@ -228,6 +229,14 @@ void launch_F_typed(lbm_grid* g, int L, int64_t k, int kind) {
     }
     launch_coalesce(g->Q, g->prec, g->dev[L + 1].pop[1], g->dev[L + 1].pop[0], g->dev[L].pop[k & 1],
                     g->dev[L].coal_fill, g->dev[L].coal_cand, (int32_t)(H.coal_fill.size() / 2), g->stream);
+  }
+  if (g->sched & LBM_SCHED_UNFUSED) {  // S_L^k then C_L^{k+1} in place (fusion ablation)
+    launch_level_step(g->Q, g->coll, g->prec, 3, &p, g->stream);
+    StepParams<T> c = p;
+    c.src = p.dst;
+    c.nghost = 0;
+    launch_level_step(g->Q, g->coll, g->prec, 4, &c, g->stream);
+    return;
   }
   launch_level_step(g->Q, g->coll, g->prec, 0, &p, g->stream);
 }
@@ -448,7 +457,9 @@ static void fill_info(const std::vector<HostLevel>& host, int Q, int prec, lbm_g
   info->Q = Q;
   info->precision = prec;
   info->kernels_per_step = (1 << host.size()) - 1;
+  info->launches_per_step = info->kernels_per_step;
   for (size_t L = 0; L < host.size(); ++L) {
+    if (!host[L].coal_fill.empty()) info->launches_per_step += (int64_t)1 << L;
     info->leaves[L] = host[L].leaves;
     info->blocks[L] = host[L].nfluid;
     info->special_blocks[L] = host[L].nspecial;
@@ -682,7 +693,7 @@ lbm_status lbm_step(lbm_grid* g, int32_t n) {
   lbm_status s;
   if (g->needs_prologue && (s = run_prologue(g))) { g->broken = true; return s; }
   if (getenv("LBMR_DEBUG_PROLOGUE_ONLY")) return LBM_OK;
-  if (getenv("LBMR_DEBUG_NO_GRAPH")) {
+  if ((g->sched & LBM_SCHED_NO_GRAPH) || getenv("LBMR_DEBUG_NO_GRAPH")) {
     std::vector<std::pair<int, int64_t>> order;
     for (int i = 0; i < n; ++i) {
       step_order(g->levels, g->steps, order);
@@ -702,6 +713,119 @@ lbm_status lbm_step(lbm_grid* g, int32_t n) {
     ++g->steps;
   }
   g->init_locked = true;
+  return LBM_OK;
+}
+
+lbm_status lbm_set_schedule(lbm_grid* g, int32_t mode) {
+  g_err.clear();
+  if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  if (mode < 0 || mode > (LBM_SCHED_UNFUSED | LBM_SCHED_NO_GRAPH)) return fail(LBM_E_INVAL, "bad schedule mode");
+  if ((mode & LBM_SCHED_UNFUSED) && g->n_ranks > 1)
+    return fail(LBM_E_UNSUPPORTED, "the unfused schedule is single-rank only");
+  if (mode == g->sched) return LBM_OK;
+  CUDA_TRY(cudaStreamSynchronize(g->stream));
+  for (int p = 0; p < 2; ++p)
+    if (g->graph[p]) {
+      cudaGraphExecDestroy(g->graph[p]);
+      g->graph[p] = nullptr;
+    }
+  g->sched = mode;
+  return LBM_OK;
+}
+
+// ---- checkpoint / resume --------------------------------------------------
+// Layout: CkptHeader, then per level the current population buffer
+// (post-collision state C_L^{k+1} incl. its explosion/coalescence ghosts, or
+// the initial post-streaming state before the first step).  At a coarse-step
+// boundary nothing else is live: every other buffer is rewritten before it is
+// read in the next step, which the resume tests check bitwise.
+namespace {
+struct CkptHeader {
+  uint32_t magic, version;
+  int32_t levels, Q, coll, prec, n_ranks, rank;
+  int64_t steps;
+  int32_t needs_prologue, sched;
+  int64_t nfluid[16];
+  int64_t leaves[16];
+};
+constexpr uint32_t kCkptMagic = 0x4b434d4cu;  // "LMCK"
+}  // namespace
+
+lbm_status lbm_checkpoint_size(const lbm_grid* g, int64_t* bytes) {
+  g_err.clear();
+  if (!g || !bytes) return fail(LBM_E_INVAL, "NULL argument");
+  int64_t n = sizeof(CkptHeader);
+  for (int L = 0; L < g->levels; ++L) n += (int64_t)pop_bytes(g, L);
+  *bytes = n;
+  return LBM_OK;
+}
+
+lbm_status lbm_checkpoint_save(lbm_grid* g, void* host, int64_t capacity) {
+  g_err.clear();
+  if (!g || !host) return fail(LBM_E_INVAL, "NULL argument");
+  if (g->broken) return fail(LBM_E_STATE, "grid is in an error state");
+  int64_t need = 0;
+  lbm_checkpoint_size(g, &need);
+  if (capacity < need) return fail(LBM_E_INVAL, "checkpoint buffer too small");
+  CkptHeader h;
+  std::memset(&h, 0, sizeof(h));
+  h.magic = kCkptMagic;
+  h.version = 1;
+  h.levels = g->levels;
+  h.Q = g->Q;
+  h.coll = g->coll;
+  h.prec = g->prec;
+  h.n_ranks = g->n_ranks;
+  h.rank = g->rank;
+  h.steps = g->steps;
+  h.needs_prologue = g->needs_prologue ? 1 : 0;
+  h.sched = g->sched;
+  for (int L = 0; L < g->levels; ++L) {
+    h.nfluid[L] = g->host[L].nfluid;
+    h.leaves[L] = g->host[L].leaves;
+  }
+  char* out = static_cast<char*>(host);
+  std::memcpy(out, &h, sizeof(h));
+  int64_t off = sizeof(h);
+  CUDA_TRY(cudaStreamSynchronize(g->stream));
+  for (int L = 0; L < g->levels; ++L) {
+    const size_t b = pop_bytes(g, L);
+    CUDA_TRY(cudaMemcpyAsync(out + off, g->dev[L].pop[cur_buf(g, L)], b, cudaMemcpyDeviceToHost, g->stream));
+    off += (int64_t)b;
+  }
+  CUDA_TRY(cudaStreamSynchronize(g->stream));
+  return LBM_OK;
+}
+
+lbm_status lbm_checkpoint_load(lbm_grid* g, const void* host, int64_t size) {
+  g_err.clear();
+  if (!g || !host) return fail(LBM_E_INVAL, "NULL argument");
+  if (g->broken) return fail(LBM_E_STATE, "grid is in an error state");
+  if (size < (int64_t)sizeof(CkptHeader)) return fail(LBM_E_INVAL, "checkpoint too small");
+  CkptHeader h;
+  std::memcpy(&h, host, sizeof(h));
+  if (h.magic != kCkptMagic || h.version != 1) return fail(LBM_E_INVAL, "not a checkpoint");
+  if (h.levels != g->levels || h.Q != g->Q || h.coll != g->coll || h.prec != g->prec || h.n_ranks != g->n_ranks ||
+      h.rank != g->rank)
+    return fail(LBM_E_INVAL, "checkpoint belongs to a different grid (levels/lattice/collision/precision/rank)");
+  for (int L = 0; L < g->levels; ++L)
+    if (h.nfluid[L] != g->host[L].nfluid || h.leaves[L] != g->host[L].leaves)
+      return fail(LBM_E_INVAL, "checkpoint grid layout differs at level " + std::to_string(L));
+  int64_t need = 0;
+  lbm_checkpoint_size(g, &need);
+  if (size < need) return fail(LBM_E_INVAL, "checkpoint truncated");
+  CUDA_TRY(cudaStreamSynchronize(g->stream));
+  g->steps = h.steps;
+  g->needs_prologue = h.needs_prologue != 0;
+  const char* in = static_cast<const char*>(host);
+  int64_t off = sizeof(h);
+  for (int L = 0; L < g->levels; ++L) {
+    const size_t b = pop_bytes(g, L);
+    CUDA_TRY(cudaMemcpyAsync(g->dev[L].pop[cur_buf(g, L)], in + off, b, cudaMemcpyHostToDevice, g->stream));
+    off += (int64_t)b;
+  }
+  CUDA_TRY(cudaStreamSynchronize(g->stream));
+  g->init_locked = h.steps > 0;
   return LBM_OK;
 }
 

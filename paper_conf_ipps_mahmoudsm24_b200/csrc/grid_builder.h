@@ -22,8 +22,7 @@ struct HostLevel {
   std::vector<uint8_t> types;    // [nblocks*512] cell type (lattice.h codes), local = x+8y+64z
   std::vector<int32_t> nbr;      // [nfluid*kRec] block records (lattice.h: neighbours, slot, origin)
   std::vector<int32_t> special_slot;  // [nfluid] index into cellinfo or -1 (plain block)
-  std::vector<uint32_t> cellinfo;     // [nspecial*512][2]: {bit q = slow link q, bit31 = fluid leaf;
-                                      //  index of the cell's first slow-link record}
+  std::vector<uint32_t> cellinfo;     // [nspecial*512][kCellInfoWords] (lattice.h)
   std::vector<uint32_t> links;        // [nlinks][2] slow-link records (lattice.h kLink*)
   std::vector<uint32_t> coal;         // coalescence candidate population indices
   int64_t nlinks = 0;

@@ -29,7 +29,7 @@ struct StepParams {
   LevelView own, coarse, fine;
   const int32_t* nbr;           // [nfluid][kRec] block records (lattice.h)
   const int32_t* special_slot;  // [nfluid]
-  const uint2* cellinfo;        // [nspecial][512] {slow-link mask | fluid bit, first link record}
+  const uint4* cellinfo;        // [nspecial][512] lattice.h kCellInfoWords layout
   const uint2* links;           // slow-link records (lattice.h kLink*)
   const uint32_t* coal;         // coalescence candidate lists
   const int32_t* origin;        // [nblocks][3] block coordinates
@@ -73,9 +73,9 @@ void launch_halo_wait(const unsigned long long* flags, int nb0, int nb1, cudaStr
 // Force-load every kernel (see level_step.cu).
 void preload_kernels();
 
-// kind: 0 = fused stream+collide over the plain blocks in ids, 1 = collide only
-// over all fluid blocks (prologue C_L^1), 2 = fused stream+collide over the
-// special blocks in ids
+// kind: 0 = fused stream+collide F_L^k, 1 = collide only (prologue C_L^1,
+// src -> dst), 3 = stream only S_L^k (unfused schedule, with the explosion
+// ghost refresh), 4 = collide dst in place (unfused schedule)
 void launch_level_step(int Q, int collision, int precision, int kind, const void* params, cudaStream_t s);
 
 // g = f^eq(rho,u) - w on the fluid cells of `nfluid` blocks; rho/u compact

@@ -51,6 +51,18 @@ constexpr int kRecOrigin = 28;
 constexpr int kRecFluid = 32;
 constexpr int kRecSpecial = 48;
 
+// per-cell info of a special block (uint4):
+//  [0] bit q = link q resolved through a slow-link record, bit 31 = fluid leaf
+//  [1] index of the cell's first slow-link record
+//  [2] bounce mask: bit q = link q is a boundary link of the cell's BC source
+//      (halfway bounce-back of the cell's own opposite population, + the
+//      moving-wall term for VELOCITY, 0 (f = w) for OUTFLOW), handled inline
+//  [3] BC source: a BC class id (< 256), kFaceSourceBase + outside pattern
+//      (class from the face table), or kNoBCSource
+constexpr int kCellInfoWords = 4;
+constexpr unsigned kFaceSourceBase = 256;
+constexpr unsigned kNoBCSource = 0xffffffffu;
+
 // slow-link record {w0, w1}: tag = w1 >> 28
 //  kLinkSame   w0 = population index at level L (irregular same-level source)
 //  kLinkCoarse w0 = population index at level L-1 (Explosion, Eq.10)

@@ -139,6 +139,18 @@ __device__ __forceinline__ double recip<double>(double x) {
   return __drcp_rn(x);
 }
 
+// Register-lean form: g^eq is never stored.  It is recomputed from (δρ, j)
+// in each of the three passes that need it (f^neq, the entropic products,
+// the update); opaque copies of the moments (fresh()) stop the compiler from
+// merging the passes' recomputations back into 27 live registers, so the
+// live set is the 27 f^neq plus a few scalars (occupancy).
+template <typename T>
+__device__ __forceinline__ T fresh(T x) {
+  if constexpr (sizeof(T) == 4) asm volatile("" : "+f"(x));
+  else asm volatile("" : "+d"(x));
+  return x;
+}
+
 template <typename T>
 __device__ __forceinline__ void collide_kbc(T (&g)[27], T omega) {
   constexpr int Q = 27;
@@ -153,35 +165,37 @@ __device__ __forceinline__ void collide_kbc(T (&g)[27], T omega) {
     if (ez(q) > 0) jz += df; else if (ez(q) < 0) jz -= df;
   }
   const T inv = recip<T>(T(1) + drho);
-  const T base = drho - T(1.5) * (jx * jx + jy * jy + jz * jz) * inv;  // g^eq = w (base + 3 e.j + 4.5 (e.j)^2 / rho)
-  const T c45 = T(4.5) * inv;
-  T geq[Q];
-  geq[0] = T(weight<Q>(0)) * base;
-#pragma unroll
-  for (int q = 1; q < Q; q += 2) {
+  const T base0 = drho - T(1.5) * (jx * jx + jy * jy + jz * jz) * inv;  // g^eq = w (base + 3 e.j + 4.5 (e.j)^2 / rho)
+  const T c450 = T(4.5) * inv;
+  // g^eq of the pair (q, q+1): sym ± asym
+  auto geq_pair = [](int q, T base, T c45, T x, T y, T z, T& sym, T& asym) {
     T ej = T(0);
-    if (ex(q) > 0) ej += jx; else if (ex(q) < 0) ej -= jx;
-    if (ey(q) > 0) ej += jy; else if (ey(q) < 0) ej -= jy;
-    if (ez(q) > 0) ej += jz; else if (ez(q) < 0) ej -= jz;
+    if (ex(q) > 0) ej += x; else if (ex(q) < 0) ej -= x;
+    if (ey(q) > 0) ej += y; else if (ey(q) < 0) ej -= y;
+    if (ez(q) > 0) ej += z; else if (ez(q) < 0) ej -= z;
     const T w = T(weight<Q>(q));
-    const T sym = w * (base + c45 * ej * ej);
-    const T asym = w * T(3) * ej;
-    geq[q] = sym + asym;
-    geq[q + 1] = sym - asym;
-  }
+    sym = w * (base + c45 * ej * ej);
+    asym = w * T(3) * ej;
+  };
+  // pass 1: f^neq in place, second moments of f^neq from pair sums
   T pxx = 0, pyy = 0, pzz = 0, pxy = 0, pxz = 0, pyz = 0;
-  g[0] -= geq[0];
+  {
+    const T base = fresh(base0), c45 = fresh(c450), x = fresh(jx), y = fresh(jy), z = fresh(jz);
+    g[0] -= T(weight<Q>(0)) * base;
 #pragma unroll
-  for (int q = 1; q < Q; q += 2) {
-    g[q] -= geq[q];
-    g[q + 1] -= geq[q + 1];
-    const T ps = g[q] + g[q + 1];
-    if (ex(q)) pxx += ps;
-    if (ey(q)) pyy += ps;
-    if (ez(q)) pzz += ps;
-    if (ex(q) * ey(q) > 0) pxy += ps; else if (ex(q) * ey(q) < 0) pxy -= ps;
-    if (ex(q) * ez(q) > 0) pxz += ps; else if (ex(q) * ez(q) < 0) pxz -= ps;
-    if (ey(q) * ez(q) > 0) pyz += ps; else if (ey(q) * ez(q) < 0) pyz -= ps;
+    for (int q = 1; q < Q; q += 2) {
+      T sym, asym;
+      geq_pair(q, base, c45, x, y, z, sym, asym);
+      g[q] -= sym + asym;
+      g[q + 1] -= sym - asym;
+      const T ps = g[q] + g[q + 1];
+      if (ex(q)) pxx += ps;
+      if (ey(q)) pyy += ps;
+      if (ez(q)) pzz += ps;
+      if (ex(q) * ey(q) > 0) pxy += ps; else if (ex(q) * ey(q) < 0) pxy -= ps;
+      if (ex(q) * ez(q) > 0) pxz += ps; else if (ex(q) * ez(q) < 0) pxz -= ps;
+      if (ey(q) * ez(q) > 0) pyz += ps; else if (ey(q) * ez(q) < 0) pyz -= ps;
+    }
   }
   const T nxz = pxx - pzz, nyz = pyy - pzz;
   const T sx = (T(2) * nxz - nyz) / T(6), sy = (-nxz + T(2) * nyz) / T(6), sz = (-nxz - nyz) / T(6);
@@ -196,22 +210,44 @@ __device__ __forceinline__ void collide_kbc(T (&g)[27], T omega) {
     }
     return T(0);
   };
+  // pass 2: <Δs|Δh>, <Δh|Δh> with weights 1/f^eq
   T sh = 0, hh = 0;
+  {
+    const T base = fresh(base0), c45 = fresh(c450), x = fresh(jx), y = fresh(jy), z = fresh(jz);
+    {
+      const T ifeq = recip<T>(T(weight<Q>(0)) * (T(1) + base));
+      const T h = g[0];
+      hh += h * h * ifeq;
+    }
 #pragma unroll
-  for (int q = 0; q < Q; ++q) {
-    const T ifeq = recip<T>(T(weight<Q>(q)) + geq[q]);
-    const T s = ds(q);
-    const T h = g[q] - s;
-    sh += s * h * ifeq;
-    hh += h * h * ifeq;
+    for (int q = 1; q < Q; q += 2) {
+      T sym, asym;
+      geq_pair(q, base, c45, x, y, z, sym, asym);
+      const T wq = T(weight<Q>(q));
+      const T i0 = recip<T>(wq + (sym + asym)), i1 = recip<T>(wq + (sym - asym));
+      const T s0 = ds(q), s1 = ds(q + 1);
+      const T h0 = g[q] - s0, h1 = g[q + 1] - s1;
+      sh += s0 * h0 * i0;
+      hh += h0 * h0 * i0;
+      sh += s1 * h1 * i1;
+      hh += h1 * h1 * i1;
+    }
   }
   const T beta = omega / T(2);
   const T gamma = (hh < T(1e-30)) ? T(2) : T(1) / beta - (T(2) - T(1) / beta) * sh / hh;
+  // pass 3: f* = f^eq + f^neq - β (2 Δs + γ Δh)
+  {
+    const T base = fresh(base0), c45 = fresh(c450), x = fresh(jx), y = fresh(jy), z = fresh(jz);
+    g[0] = T(weight<Q>(0)) * base + g[0] - beta * (gamma * g[0]);
 #pragma unroll
-  for (int q = 0; q < Q; ++q) {
-    const T s = ds(q);
-    const T h = g[q] - s;
-    g[q] = (geq[q] + g[q]) - beta * (T(2) * s + gamma * h);
+    for (int q = 1; q < Q; q += 2) {
+      T sym, asym;
+      geq_pair(q, base, c45, x, y, z, sym, asym);
+      const T s0 = ds(q), s1 = ds(q + 1);
+      const T h0 = g[q] - s0, h1 = g[q + 1] - s1;
+      g[q] = (sym + asym) + g[q] - beta * (T(2) * s0 + gamma * h0);
+      g[q + 1] = (sym - asym) + g[q + 1] - beta * (T(2) * s1 + gamma * h1);
+    }
   }
 }
 
@@ -386,19 +422,75 @@ __device__ __forceinline__ void st_pop(T* p, T v) {
 // resolve_slow; the source memory always exists).
 template <int Q, typename T, bool PRED, int q>
 __device__ __forceinline__ void pull_one(T (&g)[Q], const T* __restrict__ src, const PullGeom& G, int rec, int blk,
-                                         bool fluid) {
+                                         bool fluid, uint32_t bounce, unsigned own) {
   constexpr unsigned FULL = 0xffffffffu;
   const int nb = (q == 0) ? blk : __shfl_sync(FULL, rec, G.slot<q>());
   const unsigned off = (unsigned)nb * (unsigned)(Q * kCells) + (unsigned)G.local<q>();
   const T* p = src + q * kCells;  // constant part folds into the load's immediate offset
-  if (PRED) g[q] = (fluid && nb >= 0) ? ld_pop<T>(p + off) : T(0);
-  else g[q] = ld_pop<T>(p + off);
+  if (PRED) {
+    g[q] = (fluid && nb >= 0) ? ld_pop<T>(p + off) : T(0);
+  } else {
+    g[q] = ld_pop<T>(p + off);
+  }
 }
 
 template <int Q, typename T, bool PRED, int... qs>
 __device__ __forceinline__ void pull_all(T (&g)[Q], const T* __restrict__ src, const PullGeom& G, int rec, int blk,
-                                         bool fluid, std::integer_sequence<int, qs...>) {
-  (pull_one<Q, T, PRED, qs>(g, src, G, rec, blk, fluid), ...);
+                                         bool fluid, uint32_t bounce, unsigned own, std::integer_sequence<int, qs...>) {
+  (pull_one<Q, T, PRED, qs>(g, src, G, rec, blk, fluid, bounce, own), ...);
+}
+
+// Boundary links of the cell's BC source (bounce mask): NOSLIP keeps the
+// bounced value, VELOCITY adds 6 w_q rho_w e_q.u_w (rho_w = 1, R-A11),
+// OUTFLOW sets f_q = w_q, i.e. g_q = 0.
+// The links of the bounce mask (lattice.h cellinfo [2]) were pulled
+// speculatively from the block arithmetic's source.  bounce_issue() fetches
+// the cell's own post-collision opposite populations (halfway bounce-back,
+// P:L264) with cp.async straight into this thread's column of the shared
+// staging buffer — all in flight together and without holding registers
+// while the main pulls are in flight; apply_bounce() merges them and adds
+// the BC term.
+template <int Q, typename T>
+__device__ __forceinline__ void bounce_issue(const StepParams<T>& P, uint32_t bounce, unsigned own) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  const unsigned sv = (unsigned)__cvta_generic_to_shared(reinterpret_cast<T*>(smem_raw) + threadIdx.x);
+#pragma unroll
+  for (int q = 1; q < Q; ++q) {
+    if ((bounce >> q) & 1u) {
+      const T* a = P.src + opp(q) * kCells + own;
+      asm volatile("cp.async.ca.shared.global [%0], [%1], %2;" ::"r"(sv + (unsigned)(q * 256 * sizeof(T))), "l"(a),
+                   "n"(sizeof(T))
+                   : "memory");
+    }
+  }
+  asm volatile("cp.async.commit_group;" ::: "memory");
+}
+
+template <int Q, typename T>
+__device__ __forceinline__ void apply_bounce(const StepParams<T>& P, T (&g)[Q], uint32_t bounce, unsigned key) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  const T* sv = reinterpret_cast<const T*>(smem_raw) + threadIdx.x;
+  asm volatile("cp.async.wait_all;" ::: "memory");
+#pragma unroll
+  for (int q = 1; q < Q; ++q)
+    if ((bounce >> q) & 1u) g[q] = sv[q * 256];
+  const unsigned cls = key < kFaceSourceBase ? key : (unsigned)__ldg(P.face_cls + (key - kFaceSourceBase));
+  const int kind = __ldg(&P.bc[cls].kind);
+  if (kind == LBM_BC_NOSLIP) return;
+  if (kind == LBM_BC_OUTFLOW) {
+#pragma unroll
+    for (int q = 1; q < Q; ++q)
+      if ((bounce >> q) & 1u) g[q] = T(0);
+    return;
+  }
+  const double ux = __ldg(&P.bc[cls].u[0]), uy = __ldg(&P.bc[cls].u[1]), uz = __ldg(&P.bc[cls].u[2]);
+#pragma unroll
+  for (int q = 1; q < Q; ++q) {
+    if ((bounce >> q) & 1u) {
+      const double eu = ex(q) * ux + ey(q) * uy + ez(q) * uz;
+      g[q] += T(6.0 * weight<Q>(q) * 1.0 * eu);
+    }
+  }
 }
 
 template <int Q, typename T>
@@ -429,10 +521,10 @@ __host__ __device__ constexpr int ghost_ctas(int n) { return (n + 255) / 256; }
 #define LBMR_OCC_Q19F 6
 #endif
 #ifndef LBMR_OCC_KBCF
-#define LBMR_OCC_KBCF 2
+#define LBMR_OCC_KBCF 4
 #endif
 #ifndef LBMR_OCC_KBCD
-#define LBMR_OCC_KBCD 1
+#define LBMR_OCC_KBCD 2
 #endif
 template <int Q, typename T, int COLL = LBM_BGK>
 struct PlainOcc {
@@ -498,7 +590,9 @@ __device__ __forceinline__ void halo_store(const StepParams<T>& P, const T (&g)[
 // Other warps load the same way for their fluid cells, and the few cells with
 // slow links then apply their link records.  Offsets are 32-bit
 // (host-checked: nblocks * Q * 512 < 2^32).
-template <int Q, int COLL, typename T, bool HALO>
+// COLLIDE = false: the stream-only half S_L^k of the unfused schedule
+// (lbm_set_schedule): the pulled post-streaming populations are stored as is.
+template <int Q, int COLL, typename T, bool HALO, bool COLLIDE = true>
 __device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t) {
   constexpr unsigned FULL = 0xffffffffu;
   const int lane = threadIdx.x & 31;
@@ -508,9 +602,10 @@ __device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t
   const uint32_t sm = (uint32_t)__ldg(R + kRecSpecial + (t >> 5));
   const PullGeom G(t);
   T g[Q];
+  const unsigned own = (unsigned)blk * (unsigned)(Q * kCells) + (unsigned)t;
   if (fm == FULL && sm == 0u) {
-    pull_all<Q, T, false>(g, P.src, G, rec, blk, true, std::make_integer_sequence<int, Q>{});
-    collide<Q, COLL, T>(g, P.omega);
+    pull_all<Q, T, false>(g, P.src, G, rec, blk, true, 0u, own, std::make_integer_sequence<int, Q>{});
+    if (COLLIDE) collide<Q, COLL, T>(g, P.omega);
     store_cell<Q, T>(g, P.dst, blk, t);
     if (HALO) halo_store<Q, T>(P, g, blk, t);
     return;
@@ -518,24 +613,34 @@ __device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t
   const int slot = __shfl_sync(FULL, rec, kRecSlot);
   const bool fluid = (fm >> lane) & 1u;
   const bool special = (sm >> lane) & 1u;
-  uint2 ci = make_uint2(0u, 0u);
+  uint4 ci = make_uint4(0u, 0u, 0u, kNoBCSource);
   if (special) ci = __ldg(P.cellinfo + (unsigned)slot * kCells + t);
-  pull_all<Q, T, true>(g, P.src, G, rec, blk, fluid, std::make_integer_sequence<int, Q>{});
+  pull_all<Q, T, true>(g, P.src, G, rec, blk, fluid, 0u, own, std::make_integer_sequence<int, Q>{});
   if (!fluid) return;
-  if (special) resolve_slow<Q, T>(P, g, ci.x & ((1u << Q) - 1u), ci.y, blk, t);
-  collide<Q, COLL, T>(g, P.omega);
+#ifndef LBMR_DEBUG_NOSLOW
+  if (ci.z) bounce_issue<Q, T>(P, ci.z, own);
+  if (ci.z) apply_bounce<Q, T>(P, g, ci.z, ci.w);
+  const uint32_t recs = ci.x & ((1u << Q) - 1u);
+  if (recs) resolve_slow<Q, T>(P, g, recs, ci.y, blk, t);
+#endif
+  if (COLLIDE) collide<Q, COLL, T>(g, P.omega);
   store_cell<Q, T>(g, P.dst, blk, t);
   if (HALO) halo_store<Q, T>(P, g, blk, t);
 }
 
-// Prologue C_L^1: collision of the initial state.
-template <int Q, int COLL, typename T, bool HALO>
+// Prologue C_L^1: collision of the initial state.  INPLACE: the collide-only
+// half C_L^{k+1} of the unfused schedule, src == dst (each thread reads its
+// own cell before overwriting it, so plain loads instead of ld.global.nc).
+template <int Q, int COLL, typename T, bool HALO, bool INPLACE = false>
 __device__ __forceinline__ void collide_cell(const StepParams<T>& P, int blk, int t) {
   const uint32_t fm = (uint32_t)__ldg(P.nbr + blk * kRec + kRecFluid + (t >> 5));
   if (!((fm >> (threadIdx.x & 31)) & 1u)) return;
   T g[Q];
 #pragma unroll
-  for (int q = 0; q < Q; ++q) g[q] = __ldg(P.src + ((unsigned)blk * Q + q) * kCells + t);
+  for (int q = 0; q < Q; ++q) {
+    const T* a = P.src + ((unsigned)blk * Q + q) * kCells + t;
+    g[q] = INPLACE ? *a : __ldg(a);
+  }
   collide<Q, COLL, T>(g, P.omega);
   store_cell<Q, T>(g, P.dst, blk, t);
   if (HALO) halo_store<Q, T>(P, g, blk, t);
@@ -599,6 +704,26 @@ __global__ void __launch_bounds__(256) level_collide(const StepParams<T> P) {
     return;
   }
   collide_cell<Q, COLL, T, false>(P, blockIdx.x >> 1, ((blockIdx.x & 1) << 8) | threadIdx.x);
+}
+
+// Unfused schedule (fusion ablation, Fig.4 / Fig.9): S_L^k pulls
+// (streaming, Explosion ghosts, Coalescence ghosts, BC) into dst without
+// colliding; C_L^{k+1} then collides dst in place.  Same arithmetic as the
+// fused F_L^k, so the result is bitwise identical; it moves 4Q values per
+// leaf instead of 2Q.
+template <int Q, typename T>
+__global__ void __launch_bounds__(256, PlainOcc<Q, T, LBM_BGK>::value) level_stream(const StepParams<T> P) {
+  const int main = 2 * P.nfluid;
+  if ((int)blockIdx.x >= main) {
+    ghost_fill_one<Q, T>(P, ((int)blockIdx.x - main) * 256 + threadIdx.x);
+    return;
+  }
+  step_cell<Q, LBM_BGK, T, false, false>(P, blockIdx.x >> 1, ((blockIdx.x & 1) << 8) | threadIdx.x);
+}
+
+template <int Q, int COLL, typename T>
+__global__ void __launch_bounds__(256) level_collide_inplace(const StepParams<T> P) {
+  collide_cell<Q, COLL, T, false, true>(P, blockIdx.x >> 1, ((blockIdx.x & 1) << 8) | threadIdx.x);
 }
 
 // ---------------------------------------------------------------- init / macroscopic
@@ -719,6 +844,10 @@ static void launch_typed(int kind, const void* params, cudaStream_t s) {
   if (p.nfluid <= 0 && p.nghost <= 0) return;
   if (kind == 1) {
     level_collide<Q, COLL, T><<<dim3(2 * p.nfluid + gc), block, 0, s>>>(p);
+  } else if (kind == 3) {
+    level_stream<Q, T><<<dim3(2 * p.nfluid + gc), block, sm, s>>>(p);
+  } else if (kind == 4) {
+    if (p.nfluid > 0) level_collide_inplace<Q, COLL, T><<<dim3(2 * p.nfluid), block, 0, s>>>(p);
   } else {
     const int gct = (p.nghost + kStepThreads - 1) / kStepThreads;
     level_step_all<Q, COLL, T><<<dim3(p.nfluid * 512 / kStepThreads + gct), dim3(kStepThreads), sm, s>>>(p);
@@ -735,7 +864,10 @@ static void preload_variant() {
                        (int)slow_smem<Q, T>());
   cudaFuncSetAttribute(level_step_halo<Q, COLL, T, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                        (int)slow_smem<Q, T>());
+  cudaFuncSetAttribute(level_stream<Q, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)slow_smem<Q, T>());
   cudaFuncAttributes a;
+  cudaFuncGetAttributes(&a, level_stream<Q, T>);
+  cudaFuncGetAttributes(&a, level_collide_inplace<Q, COLL, T>);
   cudaFuncGetAttributes(&a, level_step_all<Q, COLL, T>);
   cudaFuncGetAttributes(&a, level_collide<Q, COLL, T>);
   cudaFuncGetAttributes(&a, level_step_halo<Q, COLL, T, true>);

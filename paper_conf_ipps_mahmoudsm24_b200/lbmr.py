@@ -22,6 +22,7 @@ D3Q19, D3Q27 = 19, 27
 BGK, KBC = 0, 1
 FP32, FP64 = 0, 1
 BC_NOSLIP, BC_VELOCITY, BC_OUTFLOW = 0, 1, 2
+SCHED_FUSED, SCHED_UNFUSED, SCHED_NO_GRAPH = 0, 1, 2
 
 
 class LBMError(RuntimeError):
@@ -50,6 +51,7 @@ class GridInfo(ctypes.Structure):
         ("special_blocks", ctypes.c_int64 * 16), ("special_cells", ctypes.c_int64 * 16),
         ("total_blocks", ctypes.c_int64 * 16),
         ("device_bytes", ctypes.c_int64), ("steps_done", ctypes.c_int64),
+        ("launches_per_step", ctypes.c_int64),
     ]
 
 
@@ -57,7 +59,8 @@ EXPORTS = ["lbm_grid_create", "lbm_set_bc", "lbm_init_equilibrium", "lbm_init_un
            "lbm_macroscopic", "lbm_stats", "lbm_grid_get_info", "lbm_profile_levels", "lbm_synchronize",
            "lbm_grid_destroy", "lbm_last_error", "lbm_version", "lbm_grid_analyze", "lbm_schedule",
            "lbm_lattice_table", "lbm_omega_level", "lbm_partition_cuts", "lbm_grid_slab", "lbm_halo_export",
-           "lbm_halo_connect", "lbm_halo_connect_local", "lbm_halo_plan"]
+           "lbm_halo_connect", "lbm_halo_connect_local", "lbm_halo_plan", "lbm_set_schedule",
+           "lbm_checkpoint_size", "lbm_checkpoint_save", "lbm_checkpoint_load"]
 
 _lib = None
 
@@ -103,6 +106,10 @@ def load_library(path: str = LIB_PATH):
     lib.lbm_halo_connect_local.argtypes = [P, ctypes.c_int32, P]
     lib.lbm_halo_plan.argtypes = [ctypes.POINTER(GridDesc), ctypes.c_int32, PP, ctypes.c_int32, ctypes.c_int32, lp, lp,
                                   ctypes.c_int64, lp, lp]
+    lib.lbm_set_schedule.argtypes = [P, ctypes.c_int32]
+    lib.lbm_checkpoint_size.argtypes = [P, lp]
+    lib.lbm_checkpoint_save.argtypes = [P, ctypes.c_void_p, ctypes.c_int64]
+    lib.lbm_checkpoint_load.argtypes = [P, ctypes.c_void_p, ctypes.c_int64]
     lib.lbm_last_error.restype = ctypes.c_char_p
     lib.lbm_version.restype = ctypes.c_char_p
     for name in EXPORTS:
@@ -328,6 +335,25 @@ class Grid:
         gi = GridInfo()
         _check(self.lib.lbm_grid_get_info(self.h, ctypes.byref(gi)))
         return gi
+
+    def set_schedule(self, mode: int):
+        """SCHED_FUSED (default) | SCHED_UNFUSED | SCHED_NO_GRAPH (bit flags)."""
+        _check(self.lib.lbm_set_schedule(self.h, int(mode)))
+
+    def checkpoint_size(self) -> int:
+        n = ctypes.c_int64()
+        _check(self.lib.lbm_checkpoint_size(self.h, ctypes.byref(n)))
+        return n.value
+
+    def save_checkpoint(self) -> np.ndarray:
+        """The grid's state as a host byte array (opaque; see lbmr.h)."""
+        buf = np.empty(self.checkpoint_size(), dtype=np.uint8)
+        _check(self.lib.lbm_checkpoint_save(self.h, buf.ctypes.data, buf.nbytes))
+        return buf
+
+    def load_checkpoint(self, buf: np.ndarray):
+        buf = np.ascontiguousarray(buf, dtype=np.uint8)
+        _check(self.lib.lbm_checkpoint_load(self.h, buf.ctypes.data, buf.nbytes))
 
     def profile_levels(self, n_coarse: int):
         ms = np.zeros(self.levels)

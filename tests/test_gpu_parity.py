@@ -133,3 +133,11 @@ def test_couette_gpu_exact():
         y = (np.arange(sh[1]) + 0.5) / (1 << L)
         m = ~np.isnan(r)
         assert np.abs(u[..., 0] - (U * y / H)[None, :, None])[m].max() / U < 1e-12
+
+
+@pytest.mark.parametrize("prec", [FP64, FP32])
+def test_sphere_tab1_size1(prec):
+    """the Tab. I sphere (D3Q27 KBC, 3 levels,
+    272x192x272 finest-equivalent, Re 4000) — the paper's own workload and
+    precision (fp64), 3 coarse steps."""
+    check(I.sphere_tab1(1), 3, prec)

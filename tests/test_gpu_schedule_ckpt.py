@@ -1,0 +1,156 @@
+"""Fusion ablation schedules (lbm_set_schedule) and checkpoint / resume
+(lbm_checkpoint_*), SURVEY §8(f) rows 2 and 4.
+
+The unfused schedule (stream-only S_L^k, then in-place collision) and the
+graph-free launch path run the same arithmetic as the fused F_L^k graph, so
+they must agree BITWISE with it; a resumed run must agree bitwise with an
+uninterrupted one.  Each is also checked against the fp64 oracle once."""
+import numpy as np
+import pytest
+
+import lbm_inputs as I
+from tests._parity import TOL, errors, oracle_run
+
+pytestmark = pytest.mark.gpu
+
+FP32, FP64 = 0, 1
+
+
+def _lbmr():
+    from paper_conf_ipps_mahmoudsm24_b200 import lbmr
+    return lbmr
+
+
+def _fields(g, levels):
+    return [g.macroscopic(L) for L in range(levels)]
+
+
+def _same(a, b):
+    for (ra, ua), (rb, ub) in zip(a, b):
+        assert np.array_equal(np.isnan(ra), np.isnan(rb))
+        m = ~np.isnan(ra)
+        assert np.array_equal(ra[m], rb[m]) and np.array_equal(ua[m], ub[m])
+
+
+PROBLEMS = {
+    "cavity2r": lambda: I.cavity2("r"),
+    "random4": lambda: I.random_balanced(33, n=(9, 11, 10), levels=4, p_refine=0.5),
+    "kbc_mini": lambda: I.cavity4_kbc("mini"),
+    "tunnel_s5": lambda: I.tunnel4(scale=5),
+}
+
+
+def _run(prob, prec, steps, mode):
+    lbmr = _lbmr()
+    g = lbmr.grid_from_problem(prob, precision=prec)
+    g.set_schedule(mode)
+    g.step(steps)
+    out = _fields(g, prob.levels)
+    g.close()
+    return out
+
+
+@pytest.mark.parametrize("prec", [FP64, FP32])
+@pytest.mark.parametrize("name", list(PROBLEMS))
+def test_schedules_bitwise_equal(name, prec):
+    lbmr = _lbmr()
+    prob = PROBLEMS[name]()
+    steps = 3
+    ref = _run(prob, prec, steps, lbmr.SCHED_FUSED)
+    for mode in (lbmr.SCHED_UNFUSED, lbmr.SCHED_NO_GRAPH, lbmr.SCHED_UNFUSED | lbmr.SCHED_NO_GRAPH):
+        _same(ref, _run(prob, prec, steps, mode))
+
+
+def test_unfused_matches_oracle():
+    lbmr = _lbmr()
+    prob = I.cavity2("r")
+    ora = oracle_run(prob, 10)
+    for prec in (FP64, FP32):
+        er, eu = errors(_run(prob, prec, 10, lbmr.SCHED_UNFUSED), ora)
+        assert er <= TOL[prec] and eu <= TOL[prec], (prec, er, eu)
+
+
+def test_schedule_switch_mid_run():
+    """Switching the schedule between lbm_step calls keeps the trajectory."""
+    lbmr = _lbmr()
+    prob = I.tunnel4(scale=5)
+    ref = _run(prob, FP64, 4, lbmr.SCHED_FUSED)
+    g = lbmr.grid_from_problem(prob, precision=FP64)
+    for mode in (lbmr.SCHED_UNFUSED, lbmr.SCHED_FUSED, lbmr.SCHED_NO_GRAPH, lbmr.SCHED_UNFUSED):
+        g.set_schedule(mode)
+        g.step(1)
+    _same(ref, _fields(g, prob.levels))
+    g.close()
+
+
+def test_bad_schedule_mode():
+    lbmr = _lbmr()
+    g = lbmr.grid_from_problem(I.cavity2(), precision=FP32)
+    with pytest.raises(lbmr.LBMError):
+        g.set_schedule(7)
+    g.close()
+
+
+@pytest.mark.parametrize("prec", [FP64, FP32])
+@pytest.mark.parametrize("name", list(PROBLEMS))
+@pytest.mark.parametrize("at", [0, 1, 2])
+def test_checkpoint_resume_bitwise(name, prec, at):
+    """save after `at` coarse steps (0: before the prologue ran), restore into
+    a FRESH grid (its other buffers zero), continue: == uninterrupted run."""
+    lbmr = _lbmr()
+    prob = PROBLEMS[name]()
+    total = 5
+    ref = _run(prob, prec, total, lbmr.SCHED_FUSED)
+    g = lbmr.grid_from_problem(prob, precision=prec)
+    g.step(at)
+    ck = g.save_checkpoint()
+    assert ck.nbytes == g.checkpoint_size()
+    g.close()
+    h = lbmr.grid_from_problem(prob, precision=prec, init=False)
+    h.load_checkpoint(ck)
+    assert h.info().steps_done == at
+    h.step(total - at)
+    _same(ref, _fields(h, prob.levels))
+    h.close()
+
+
+def test_checkpoint_rejects_other_grid():
+    lbmr = _lbmr()
+    g = lbmr.grid_from_problem(I.cavity2(), precision=FP32)
+    g.step(1)
+    ck = g.save_checkpoint()
+    g.close()
+    for other in (lambda: lbmr.grid_from_problem(I.cavity2(), precision=FP64),
+                  lambda: lbmr.grid_from_problem(I.tunnel4(scale=5), precision=FP32)):
+        h = other()
+        with pytest.raises(lbmr.LBMError):
+            h.load_checkpoint(ck)
+        h.close()
+    h = lbmr.grid_from_problem(I.cavity2(), precision=FP32)
+    with pytest.raises(lbmr.LBMError):
+        h.load_checkpoint(ck[:-4])  # truncated
+    bad = ck.copy()
+    bad[:4] = 0
+    with pytest.raises(lbmr.LBMError):
+        h.load_checkpoint(bad)
+    h.close()
+
+
+def test_checkpoint_partitioned_bitwise():
+    """Each slab of a 2-slab partition checkpoints its own state; resuming
+    both into fresh slabs == uninterrupted single grid."""
+    lbmr = _lbmr()
+    prob = I.tunnel4(scale=5)
+    ref = _run(prob, FP64, 4, lbmr.SCHED_FUSED)
+    pg = lbmr.PartitionedGrid(prob, 2, precision=FP64)
+    pg.step(2)
+    pg.synchronize()
+    cks = [g.save_checkpoint() for g in pg.grids]
+    pg.close()
+    pg2 = lbmr.PartitionedGrid(prob, 2, precision=FP64)
+    for g, ck in zip(pg2.grids, cks):
+        g.load_checkpoint(ck)
+    pg2.step(2)
+    got = [pg2.macroscopic(L) for L in range(prob.levels)]
+    pg2.close()
+    _same(ref, got)

@@ -1,0 +1,7 @@
+timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_gpu_schedule_ckpt.py -m gpu -x -q 2>&1 | tail -3
+BENCH_ARGS="--config tunnel4" VARIANTS="liblbmr q19o5" bash tools/gpu_variants.sh
+BENCH_ARGS="--config sphere3" VARIANTS="liblbmr q19o5" bash tools/gpu_variants.sh
+BENCH_ARGS="--config cavity4_bgk" VARIANTS="liblbmr noslow" bash tools/gpu_variants.sh
+BENCH_ARGS="--config cavity4_kbc" VARIANTS="liblbmr kbcf3 kbcf5 noslow" bash tools/gpu_variants.sh
+BENCH_ARGS="--config cavity4_kbc --precision fp64" VARIANTS="liblbmr kbcd3" bash tools/gpu_variants.sh
+BENCH_ARGS="--config sphere_tab1_s3" VARIANTS="liblbmr kbcd3 noslow" bash tools/gpu_variants.sh
