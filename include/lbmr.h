@@ -124,6 +124,14 @@ lbm_status lbm_step(lbm_grid* g, int32_t n_coarse);
  * leaves get NaN.  Synchronises the grid's stream. */
 lbm_status lbm_macroscopic(lbm_grid* g, int32_t level, double* rho, double* u);
 
+/* Probes (also the sampled full-size parity checks):
+ * rho (Eq.6) and u (Eq.7) at n cells of level `level` given as GLOBAL
+ * level-L integer coordinates xyz[3n] (x, y, z).  rho[n] and u[3n] are
+ * caller-owned host arrays.  Cells that are outside the domain, not fluid
+ * leaves of this level, or owned by another rank of a partition get NaN.
+ * Synchronises the grid's stream. */
+lbm_status lbm_probe(lbm_grid* g, int32_t level, int64_t n, const int64_t* xyz, double* rho, double* u);
+
 /* Fluid leaves per level (leaves_per_level[levels], may be NULL) and total
  * mass sum_L sum_leaves rho * 8^-L in coarse-cell volumes (may be NULL).
  * Synchronises. */

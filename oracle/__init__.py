@@ -61,6 +61,7 @@ def _load():
         lib.ora_step.argtypes = [P, ctypes.c_int]
         lib.ora_macroscopic.argtypes = [P, ctypes.c_int, dp, dp]
         lib.ora_get_f.argtypes = [P, ctypes.c_int, dp]
+        lib.ora_probe.argtypes = [P, ctypes.c_int, ctypes.c_int64, ctypes.POINTER(ctypes.c_int64), dp, dp]
         lib.ora_set_f.argtypes = [P, ctypes.c_int, dp]
         _lib = lib
     return _lib
@@ -156,6 +157,14 @@ class Oracle:
         rho = np.empty(shape)
         u = np.empty(shape + (3,))
         self.lib.ora_macroscopic(self.h, L, _dp(rho), _dp(u))
+        return rho, u
+
+    def probe(self, L: int, xyz):
+        """(rho[n], u[n,3]) at level-L cells xyz[n,3]; NaN off fluid leaves."""
+        xyz = np.ascontiguousarray(xyz, dtype=np.int64).reshape(-1, 3)
+        rho = np.empty(len(xyz))
+        u = np.empty((len(xyz), 3))
+        self.lib.ora_probe(self.h, L, len(xyz), xyz.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)), _dp(rho), _dp(u))
         return rho, u
 
     def get_f(self, L: int):

@@ -577,7 +577,7 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
       if (cudaMemset(D.pop[b], 0, pop_bytes(g, L)) != cudaSuccess) return cleanup(fail(LBM_E_CUDA, "memset"));
     }
     // the dense per-level tables are on the device now; keep only counters
-    std::vector<int32_t>().swap(H.blkmap);
+    // (the host block map is kept for lbm_probe)
     std::vector<uint32_t>().swap(H.cellinfo);
     std::vector<uint32_t>().swap(H.links);
     std::vector<uint32_t>().swap(H.coal);
@@ -920,6 +920,46 @@ lbm_status lbm_macroscopic(lbm_grid* g, int32_t L, double* rho, double* u) {
       if (u) { u[3 * c] = v[3 * k]; u[3 * c + 1] = v[3 * k + 1]; u[3 * c + 2] = v[3 * k + 2]; }
     }
   }
+  return LBM_OK;
+}
+
+lbm_status lbm_probe(lbm_grid* g, int32_t L, int64_t n, const int64_t* xyz, double* rho, double* u) {
+  g_err.clear();
+  if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  if (L < 0 || L >= g->levels) return fail(LBM_E_INVAL, "level out of range");
+  if (n < 0 || (n > 0 && (!xyz || !rho || !u))) return fail(LBM_E_INVAL, "bad probe arguments");
+  if (n == 0) return LBM_OK;
+  const HostLevel& H = g->host[L];
+  const int64_t xoff = (int64_t)g->x_lo << L;  // global -> local x (partitioned grids)
+  const int64_t gnx = (int64_t)g->desc.nx << L;
+  std::vector<int64_t> cell(n, -1);
+#pragma omp parallel for schedule(static)
+  for (int64_t i = 0; i < n; ++i) {
+    int64_t x = xyz[3 * i], y = xyz[3 * i + 1], z = xyz[3 * i + 2];
+    if (x < 0 || x >= gnx || y < 0 || y >= H.n[1] || z < 0 || z >= H.n[2]) continue;
+    x -= xoff;
+    if (x < H.owned_lo || x >= H.owned_hi) continue;  // another rank's cell
+    const int32_t b = H.blkmap[((x >> 3) * H.nb[1] + (y >> 3)) * H.nb[2] + (z >> 3)];
+    if (b < 0 || b >= H.nlaunch) continue;
+    const int l = (int)((x & 7) + 8 * (y & 7) + 64 * (z & 7));
+    if (H.types[(size_t)b * kCells + l] != kFluid) continue;
+    cell[i] = (int64_t)b * kCells + l;
+  }
+  int64_t* dc = nullptr;
+  double *dr = nullptr, *du = nullptr;
+  CUDA_TRY(cudaStreamSynchronize(g->stream));
+  CUDA_TRY(cudaMalloc(&dc, n * sizeof(int64_t)));
+  CUDA_TRY(cudaMalloc(&dr, n * sizeof(double)));
+  CUDA_TRY(cudaMalloc(&du, 3 * n * sizeof(double)));
+  CUDA_TRY(cudaMemcpyAsync(dc, cell.data(), n * sizeof(int64_t), cudaMemcpyHostToDevice, g->stream));
+  launch_probe(g->Q, g->prec, g->dev[L].pop[cur_buf(g, L)], dc, n, dr, du, g->stream);
+  CUDA_TRY(cudaGetLastError());
+  CUDA_TRY(cudaMemcpyAsync(rho, dr, n * sizeof(double), cudaMemcpyDeviceToHost, g->stream));
+  CUDA_TRY(cudaMemcpyAsync(u, du, 3 * n * sizeof(double), cudaMemcpyDeviceToHost, g->stream));
+  CUDA_TRY(cudaStreamSynchronize(g->stream));
+  cudaFree(dc);
+  cudaFree(dr);
+  cudaFree(du);
   return LBM_OK;
 }
 

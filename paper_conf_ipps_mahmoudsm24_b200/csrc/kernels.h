@@ -66,6 +66,11 @@ struct StepParams {
 void launch_coalesce(int Q, int precision, const void* fa, const void* fb, void* dst, const uint32_t* fill,
                      const uint32_t* cand, int32_t n, cudaStream_t s);
 
+// rho / u (double) of n cells given by population cell index block*512+local
+// (-1 -> NaN), read from the post-collision buffer `pop`.
+void launch_probe(int Q, int precision, const void* pop, const int64_t* cell, int64_t n, double* rho, double* u,
+                  cudaStream_t s);
+
 // One-thread kernel: wait until both neighbours (has_nb) have completed the
 // cut-plane part of every kernel this rank has completed.
 void launch_halo_wait(const unsigned long long* flags, int nb0, int nb1, cudaStream_t s);

@@ -210,8 +210,9 @@ __device__ __forceinline__ void collide_kbc(T (&g)[27], T omega) {
     }
     return T(0);
   };
-  // pass 2: <Δs|Δh>, <Δh|Δh> with weights 1/f^eq
-  T sh = 0, hh = 0;
+  // pass 2: <Δs|Δh>, <Δh|Δh> with weights 1/f^eq (two partial sums each:
+  // shorter dependent-add chains for the fp64 pipe)
+  T sh = 0, hh = 0, sh2 = 0, hh2 = 0;
   {
     const T base = fresh(base0), c45 = fresh(c450), x = fresh(jx), y = fresh(jy), z = fresh(jz);
     {
@@ -223,16 +224,20 @@ __device__ __forceinline__ void collide_kbc(T (&g)[27], T omega) {
     for (int q = 1; q < Q; q += 2) {
       T sym, asym;
       geq_pair(q, base, c45, x, y, z, sym, asym);
-      const T wq = T(weight<Q>(q));
-      const T i0 = recip<T>(wq + (sym + asym)), i1 = recip<T>(wq + (sym - asym));
+      // one reciprocal per opposite pair: 1/(a+b) = (a-b)/(a²-b²), 1/(a-b) = (a+b)/(a²-b²)
+      const T a = T(weight<Q>(q)) + sym;
+      const T r = recip<T>(a * a - asym * asym);
+      const T i0 = (a - asym) * r, i1 = (a + asym) * r;
       const T s0 = ds(q), s1 = ds(q + 1);
       const T h0 = g[q] - s0, h1 = g[q + 1] - s1;
       sh += s0 * h0 * i0;
       hh += h0 * h0 * i0;
-      sh += s1 * h1 * i1;
-      hh += h1 * h1 * i1;
+      sh2 += s1 * h1 * i1;
+      hh2 += h1 * h1 * i1;
     }
   }
+  sh += sh2;
+  hh += hh2;
   const T beta = omega / T(2);
   const T gamma = (hh < T(1e-30)) ? T(2) : T(1) / beta - (T(2) - T(1) / beta) * sh / hh;
   // pass 3: f* = f^eq + f^neq - β (2 Δs + γ Δh)
@@ -272,14 +277,11 @@ __device__ __forceinline__ void collide(T (&g)[Q], T omega) {
 //                               in candidate order like the oracle.
 __device__ __forceinline__ int opp_rt(int q) { return q == 0 ? 0 : ((q & 1) ? q + 1 : q - 1); }
 
+// Values go to this thread's column sv[q * 256] of a shared buffer
+// (conflict-free for any q per lane).
 template <int Q, typename T>
-__device__ __forceinline__ void resolve_slow(const StepParams<T>& P, T (&g)[Q], uint32_t slow, unsigned j, int blk,
-                                             int t) {
-  // values go to this thread's column of a shared buffer sv[q][threadIdx]
-  // (conflict-free for any q per lane) and are merged once at the end
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  T* sv = reinterpret_cast<T*>(smem_raw) + threadIdx.x;
-  const uint32_t all = slow;
+__device__ __forceinline__ void resolve_slow_sv(const StepParams<T>& P, T* sv, uint32_t slow, unsigned j, int blk,
+                                                int t) {
   const unsigned own = (unsigned)blk * (unsigned)(Q * kCells) + (unsigned)t;
 #ifndef LBMR_SLOW_NB
 #define LBMR_SLOW_NB 4
@@ -337,9 +339,17 @@ __device__ __forceinline__ void resolve_slow(const StepParams<T>& P, T (&g)[Q], 
       sv[q * 256] = val;
     }
   }
+}
+
+template <int Q, typename T>
+__device__ __forceinline__ void resolve_slow(const StepParams<T>& P, T (&g)[Q], uint32_t slow, unsigned j, int blk,
+                                             int t) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  T* sv = reinterpret_cast<T*>(smem_raw) + threadIdx.x;
+  resolve_slow_sv<Q, T>(P, sv, slow, j, blk, t);
 #pragma unroll
   for (int q = 0; q < Q; ++q)
-    if (all & (1u << q)) g[q] = sv[q * 256];
+    if (slow & (1u << q)) g[q] = sv[q * 256];
 }
 
 // ---------------------------------------------------------------- fused kernel
@@ -422,7 +432,7 @@ __device__ __forceinline__ void st_pop(T* p, T v) {
 // resolve_slow; the source memory always exists).
 template <int Q, typename T, bool PRED, int q>
 __device__ __forceinline__ void pull_one(T (&g)[Q], const T* __restrict__ src, const PullGeom& G, int rec, int blk,
-                                         bool fluid, uint32_t bounce, unsigned own) {
+                                         bool fluid) {
   constexpr unsigned FULL = 0xffffffffu;
   const int nb = (q == 0) ? blk : __shfl_sync(FULL, rec, G.slot<q>());
   const unsigned off = (unsigned)nb * (unsigned)(Q * kCells) + (unsigned)G.local<q>();
@@ -436,8 +446,8 @@ __device__ __forceinline__ void pull_one(T (&g)[Q], const T* __restrict__ src, c
 
 template <int Q, typename T, bool PRED, int... qs>
 __device__ __forceinline__ void pull_all(T (&g)[Q], const T* __restrict__ src, const PullGeom& G, int rec, int blk,
-                                         bool fluid, uint32_t bounce, unsigned own, std::integer_sequence<int, qs...>) {
-  (pull_one<Q, T, PRED, qs>(g, src, G, rec, blk, fluid, bounce, own), ...);
+                                         bool fluid, std::integer_sequence<int, qs...>) {
+  (pull_one<Q, T, PRED, qs>(g, src, G, rec, blk, fluid), ...);
 }
 
 // Boundary links of the cell's BC source (bounce mask): NOSLIP keeps the
@@ -467,6 +477,9 @@ __device__ __forceinline__ void bounce_issue(const StepParams<T>& P, uint32_t bo
 }
 
 template <int Q, typename T>
+__device__ __forceinline__ void bounce_fix(const StepParams<T>& P, T (&g)[Q], uint32_t bounce, unsigned key);
+
+template <int Q, typename T>
 __device__ __forceinline__ void apply_bounce(const StepParams<T>& P, T (&g)[Q], uint32_t bounce, unsigned key) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const T* sv = reinterpret_cast<const T*>(smem_raw) + threadIdx.x;
@@ -474,6 +487,13 @@ __device__ __forceinline__ void apply_bounce(const StepParams<T>& P, T (&g)[Q], 
 #pragma unroll
   for (int q = 1; q < Q; ++q)
     if ((bounce >> q) & 1u) g[q] = sv[q * 256];
+  bounce_fix<Q, T>(P, g, bounce, key);
+}
+
+// BC term of the bounce links: NOSLIP keeps the bounced value, VELOCITY adds
+// 6 w_q rho_w e_q.u_w (rho_w = 1, R-A11), OUTFLOW sets f_q = w_q, i.e. g_q = 0.
+template <int Q, typename T>
+__device__ __forceinline__ void bounce_fix(const StepParams<T>& P, T (&g)[Q], uint32_t bounce, unsigned key) {
   const unsigned cls = key < kFaceSourceBase ? key : (unsigned)__ldg(P.face_cls + (key - kFaceSourceBase));
   const int kind = __ldg(&P.bc[cls].kind);
   if (kind == LBM_BC_NOSLIP) return;
@@ -526,11 +546,14 @@ __host__ __device__ constexpr int ghost_ctas(int n) { return (n + 255) / 256; }
 #ifndef LBMR_OCC_KBCD
 #define LBMR_OCC_KBCD 2
 #endif
+#ifndef LBMR_OCC_BGKD
+#define LBMR_OCC_BGKD 3
+#endif
 template <int Q, typename T, int COLL = LBM_BGK>
 struct PlainOcc {
   static constexpr int value = COLL == LBM_KBC ? (sizeof(T) == 4 ? LBMR_OCC_KBCF : LBMR_OCC_KBCD)
                                : (Q == 19 && sizeof(T) == 4) ? LBMR_OCC_Q19F
-                               : (sizeof(T) == 4 ? 3 : 2);
+                               : (sizeof(T) == 4 ? 3 : (Q == 19 ? LBMR_OCC_BGKD : 2));
 };
 
 // ---------------------------------------------------------------- halo protocol
@@ -603,26 +626,33 @@ __device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t
   const PullGeom G(t);
   T g[Q];
   const unsigned own = (unsigned)blk * (unsigned)(Q * kCells) + (unsigned)t;
+  // KBC: one collision / store site for both paths (half the code: fewer
+  // instruction-cache misses with the long collision); BGK: separate sites,
+  // so the plain path keeps its own spill-free register assignment
+  constexpr bool kShared = (COLL == LBM_KBC);
   if (fm == FULL && sm == 0u) {
-    pull_all<Q, T, false>(g, P.src, G, rec, blk, true, 0u, own, std::make_integer_sequence<int, Q>{});
-    if (COLLIDE) collide<Q, COLL, T>(g, P.omega);
-    store_cell<Q, T>(g, P.dst, blk, t);
-    if (HALO) halo_store<Q, T>(P, g, blk, t);
-    return;
-  }
-  const int slot = __shfl_sync(FULL, rec, kRecSlot);
-  const bool fluid = (fm >> lane) & 1u;
-  const bool special = (sm >> lane) & 1u;
-  uint4 ci = make_uint4(0u, 0u, 0u, kNoBCSource);
-  if (special) ci = __ldg(P.cellinfo + (unsigned)slot * kCells + t);
-  pull_all<Q, T, true>(g, P.src, G, rec, blk, fluid, 0u, own, std::make_integer_sequence<int, Q>{});
-  if (!fluid) return;
+    pull_all<Q, T, false>(g, P.src, G, rec, blk, true, std::make_integer_sequence<int, Q>{});
+    if (!kShared) {
+      if (COLLIDE) collide<Q, COLL, T>(g, P.omega);
+      store_cell<Q, T>(g, P.dst, blk, t);
+      if (HALO) halo_store<Q, T>(P, g, blk, t);
+      return;
+    }
+  } else {
+    const int slot = __shfl_sync(FULL, rec, kRecSlot);
+    const bool fluid = (fm >> lane) & 1u;
+    const bool special = (sm >> lane) & 1u;
+    uint4 ci = make_uint4(0u, 0u, 0u, kNoBCSource);
+    if (special) ci = __ldg(P.cellinfo + (unsigned)slot * kCells + t);
+    pull_all<Q, T, true>(g, P.src, G, rec, blk, fluid, std::make_integer_sequence<int, Q>{});
+    if (!fluid) return;
 #ifndef LBMR_DEBUG_NOSLOW
-  if (ci.z) bounce_issue<Q, T>(P, ci.z, own);
-  if (ci.z) apply_bounce<Q, T>(P, g, ci.z, ci.w);
-  const uint32_t recs = ci.x & ((1u << Q) - 1u);
-  if (recs) resolve_slow<Q, T>(P, g, recs, ci.y, blk, t);
+    if (ci.z) bounce_issue<Q, T>(P, ci.z, own);
+    if (ci.z) apply_bounce<Q, T>(P, g, ci.z, ci.w);
+    const uint32_t recs = ci.x & ((1u << Q) - 1u);
+    if (recs) resolve_slow<Q, T>(P, g, recs, ci.y, blk, t);
 #endif
+  }
   if (COLLIDE) collide<Q, COLL, T>(g, P.omega);
   store_cell<Q, T>(g, P.dst, blk, t);
   if (HALO) halo_store<Q, T>(P, g, blk, t);
@@ -789,6 +819,48 @@ __global__ void __launch_bounds__(512) macroscopic_kernel(const T* pop, const in
   }
 }
 
+// Probes: rho, u (Eq.6-7) of n cells given by their population cell index
+// block*512 + local (or -1 -> NaN).  One thread per probe.
+template <int Q, typename T>
+__global__ void __launch_bounds__(256) probe_kernel(const T* __restrict__ pop, const int64_t* __restrict__ cell,
+                                                    int64_t n, double* __restrict__ rho, double* __restrict__ u) {
+  const int64_t i = (int64_t)blockIdx.x * 256 + threadIdx.x;
+  if (i >= n) return;
+  const int64_t c = cell[i];
+  if (c < 0) {
+    rho[i] = u[3 * i] = u[3 * i + 1] = u[3 * i + 2] = NAN;
+    return;
+  }
+  const T* s = pop + (c >> 9) * (int64_t)(Q * kCells) + (c & 511);
+  double d = 0, jx = 0, jy = 0, jz = 0;
+#pragma unroll
+  for (int q = 0; q < Q; ++q) {
+    const double g = (double)s[(int64_t)q * kCells];
+    d += g;
+    jx += ex(q) * g;
+    jy += ey(q) * g;
+    jz += ez(q) * g;
+  }
+  const double r = 1.0 + d;
+  rho[i] = r;
+  u[3 * i] = jx / r;
+  u[3 * i + 1] = jy / r;
+  u[3 * i + 2] = jz / r;
+}
+
+void launch_probe(int Q, int precision, const void* pop, const int64_t* cell, int64_t n, double* rho, double* u,
+                  cudaStream_t s) {
+  if (n <= 0) return;
+  const unsigned grid = (unsigned)((n + 255) / 256);
+  if (precision == LBM_FP32) {
+    if (Q == 19) probe_kernel<19, float><<<grid, 256, 0, s>>>((const float*)pop, cell, n, rho, u);
+    else probe_kernel<27, float><<<grid, 256, 0, s>>>((const float*)pop, cell, n, rho, u);
+  } else {
+    if (Q == 19) probe_kernel<19, double><<<grid, 256, 0, s>>>((const double*)pop, cell, n, rho, u);
+    else probe_kernel<27, double><<<grid, 256, 0, s>>>((const double*)pop, cell, n, rho, u);
+  }
+}
+
 // Coalescence ghosts: one thread per (ghost cell, q) entry.
 // Fine candidates summed in candidate order, first substep then second, like
 // the oracle (Eq.11, n = 2|B|, R-A2/R-A3).
@@ -884,6 +956,10 @@ void preload_kernels() {
   cudaFuncAttributes a;
   cudaFuncGetAttributes(&a, halo_wait_kernel);
   cudaFuncGetAttributes(&a, coalesce_kernel<float>);
+  cudaFuncGetAttributes(&a, probe_kernel<19, float>);
+  cudaFuncGetAttributes(&a, probe_kernel<27, float>);
+  cudaFuncGetAttributes(&a, probe_kernel<19, double>);
+  cudaFuncGetAttributes(&a, probe_kernel<27, double>);
   cudaFuncGetAttributes(&a, coalesce_kernel<double>);
   cudaFuncGetAttributes(&a, init_eq_kernel<19, float>);
   cudaFuncGetAttributes(&a, init_eq_kernel<27, float>);

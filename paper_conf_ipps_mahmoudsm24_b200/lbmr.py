@@ -60,7 +60,7 @@ EXPORTS = ["lbm_grid_create", "lbm_set_bc", "lbm_init_equilibrium", "lbm_init_un
            "lbm_grid_destroy", "lbm_last_error", "lbm_version", "lbm_grid_analyze", "lbm_schedule",
            "lbm_lattice_table", "lbm_omega_level", "lbm_partition_cuts", "lbm_grid_slab", "lbm_halo_export",
            "lbm_halo_connect", "lbm_halo_connect_local", "lbm_halo_plan", "lbm_set_schedule",
-           "lbm_checkpoint_size", "lbm_checkpoint_save", "lbm_checkpoint_load"]
+           "lbm_checkpoint_size", "lbm_checkpoint_save", "lbm_checkpoint_load", "lbm_probe"]
 
 _lib = None
 
@@ -107,6 +107,7 @@ def load_library(path: str = LIB_PATH):
     lib.lbm_halo_plan.argtypes = [ctypes.POINTER(GridDesc), ctypes.c_int32, PP, ctypes.c_int32, ctypes.c_int32, lp, lp,
                                   ctypes.c_int64, lp, lp]
     lib.lbm_set_schedule.argtypes = [P, ctypes.c_int32]
+    lib.lbm_probe.argtypes = [P, ctypes.c_int32, ctypes.c_int64, lp, dp, dp]
     lib.lbm_checkpoint_size.argtypes = [P, lp]
     lib.lbm_checkpoint_save.argtypes = [P, ctypes.c_void_p, ctypes.c_int64]
     lib.lbm_checkpoint_load.argtypes = [P, ctypes.c_void_p, ctypes.c_int64]
@@ -322,6 +323,16 @@ class Grid:
         rho = np.empty(shape)
         u = np.empty(shape + (3,))
         _check(self.lib.lbm_macroscopic(self.h, int(L), _dp(rho), _dp(u)))
+        return rho, u
+
+    def probe(self, L: int, xyz):
+        """(rho[n], u[n,3]) at GLOBAL level-L cells xyz[n,3]; NaN off this
+        rank's fluid leaves."""
+        xyz = np.ascontiguousarray(xyz, dtype=np.int64).reshape(-1, 3)
+        rho = np.empty(len(xyz))
+        u = np.empty((len(xyz), 3))
+        _check(self.lib.lbm_probe(self.h, int(L), len(xyz), xyz.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)),
+                                  _dp(rho), _dp(u)))
         return rho, u
 
     def stats(self):
