@@ -102,6 +102,12 @@ struct lbm_grid {
   unsigned long long* flags = nullptr;      // [4], see kernels.h
   unsigned long long* peer_flags[2] = {nullptr, nullptr};
   std::vector<std::pair<std::string, void*>> ipc_open;  // opened IPC handles
+  // reusable device / pinned host scratch of the diagnostics calls
+  // (lbm_stats, lbm_probe): no allocation per call
+  void* scratch = nullptr;
+  size_t scratch_bytes = 0;
+  void* hscratch = nullptr;
+  size_t hscratch_bytes = 0;
 };
 
 namespace {
@@ -261,6 +267,38 @@ void step_order(int levels, int64_t n, std::vector<std::pair<int, int64_t>>& out
       out.push_back({L, kk});
     }
   }
+}
+
+// Scratch buffers grow on demand; every user synchronises before returning,
+// so a reallocation never races with work still reading the old buffer.
+lbm_status scratch_dev(lbm_grid* g, size_t bytes, void** out) {
+  if (g->scratch_bytes < bytes) {
+    if (g->scratch) cudaFree(g->scratch);
+    g->scratch = nullptr;
+    g->scratch_bytes = 0;
+    if (cudaMalloc(&g->scratch, bytes) != cudaSuccess) {
+      cudaGetLastError();
+      return fail(LBM_E_OOM, "cudaMalloc failed (scratch)");
+    }
+    g->scratch_bytes = bytes;
+  }
+  *out = g->scratch;
+  return LBM_OK;
+}
+
+lbm_status scratch_host(lbm_grid* g, size_t bytes, void** out) {
+  if (g->hscratch_bytes < bytes) {
+    if (g->hscratch) cudaFreeHost(g->hscratch);
+    g->hscratch = nullptr;
+    g->hscratch_bytes = 0;
+    if (cudaMallocHost(&g->hscratch, bytes) != cudaSuccess) {
+      cudaGetLastError();
+      return fail(LBM_E_OOM, "cudaMallocHost failed (scratch)");
+    }
+    g->hscratch_bytes = bytes;
+  }
+  *out = g->hscratch;
+  return LBM_OK;
 }
 
 lbm_status run_prologue(lbm_grid* g) {
@@ -945,21 +983,24 @@ lbm_status lbm_probe(lbm_grid* g, int32_t L, int64_t n, const int64_t* xyz, doub
     if (H.types[(size_t)b * kCells + l] != kFluid) continue;
     cell[i] = (int64_t)b * kCells + l;
   }
-  int64_t* dc = nullptr;
-  double *dr = nullptr, *du = nullptr;
+  // scratch layout: cell indices, then rho[n], u[3n] (device); the same
+  // through pinned host memory
+  const size_t bytes = (size_t)n * (sizeof(int64_t) + 4 * sizeof(double));
+  void *dv = nullptr, *hv = nullptr;
+  lbm_status s;
+  if ((s = scratch_dev(g, bytes, &dv)) || (s = scratch_host(g, bytes, &hv))) return s;
   CUDA_TRY(cudaStreamSynchronize(g->stream));
-  CUDA_TRY(cudaMalloc(&dc, n * sizeof(int64_t)));
-  CUDA_TRY(cudaMalloc(&dr, n * sizeof(double)));
-  CUDA_TRY(cudaMalloc(&du, 3 * n * sizeof(double)));
-  CUDA_TRY(cudaMemcpyAsync(dc, cell.data(), n * sizeof(int64_t), cudaMemcpyHostToDevice, g->stream));
-  launch_probe(g->Q, g->prec, g->dev[L].pop[cur_buf(g, L)], dc, n, dr, du, g->stream);
+  std::memcpy(hv, cell.data(), n * sizeof(int64_t));
+  int64_t* dc = static_cast<int64_t*>(dv);
+  double* dr = reinterpret_cast<double*>(dc + n);
+  double* hr = reinterpret_cast<double*>(static_cast<int64_t*>(hv) + n);
+  CUDA_TRY(cudaMemcpyAsync(dc, hv, n * sizeof(int64_t), cudaMemcpyHostToDevice, g->stream));
+  launch_probe(g->Q, g->prec, g->dev[L].pop[cur_buf(g, L)], dc, n, dr, dr + n, g->stream);
   CUDA_TRY(cudaGetLastError());
-  CUDA_TRY(cudaMemcpyAsync(rho, dr, n * sizeof(double), cudaMemcpyDeviceToHost, g->stream));
-  CUDA_TRY(cudaMemcpyAsync(u, du, 3 * n * sizeof(double), cudaMemcpyDeviceToHost, g->stream));
+  CUDA_TRY(cudaMemcpyAsync(hr, dr, 4 * n * sizeof(double), cudaMemcpyDeviceToHost, g->stream));
   CUDA_TRY(cudaStreamSynchronize(g->stream));
-  cudaFree(dc);
-  cudaFree(dr);
-  cudaFree(du);
+  std::memcpy(rho, hr, n * sizeof(double));
+  std::memcpy(u, hr + n, 3 * n * sizeof(double));
   return LBM_OK;
 }
 
@@ -969,20 +1010,31 @@ lbm_status lbm_stats(lbm_grid* g, int64_t* leaves, double* mass) {
   if (leaves)
     for (int L = 0; L < g->levels; ++L) leaves[L] = g->host[L].leaves;
   if (!mass) return LBM_OK;
-  double total = 0.0;
+  // per-block mass partial sums of every level into one scratch buffer, one
+  // D2H copy, one synchronisation
+  size_t nb = 0;
+  for (int L = 0; L < g->levels; ++L) nb += (size_t)std::max<int32_t>(g->host[L].nlaunch, 1);
+  void *dv = nullptr, *hv = nullptr;
+  lbm_status s;
+  if ((s = scratch_dev(g, nb * sizeof(double), &dv)) || (s = scratch_host(g, nb * sizeof(double), &hv))) return s;
+  double* bm = static_cast<double*>(dv);
+  size_t off = 0;
   for (int L = 0; L < g->levels; ++L) {
     const HostLevel& H = g->host[L];
-    double* bm = nullptr;
-    CUDA_TRY(cudaMalloc(&bm, std::max<int32_t>(H.nlaunch, 1) * sizeof(double)));
     launch_macroscopic(g->Q, g->prec, g->dev[L].pop[cur_buf(g, L)], g->dev[L].nbr, H.nlaunch, nullptr, nullptr,
-                       bm, g->stream);
-    std::vector<double> h(H.nlaunch);
-    CUDA_TRY(cudaGetLastError());
-    CUDA_TRY(cudaMemcpyAsync(h.data(), bm, H.nlaunch * sizeof(double), cudaMemcpyDeviceToHost, g->stream));
-    CUDA_TRY(cudaStreamSynchronize(g->stream));
-    cudaFree(bm);
+                       bm + off, g->stream);
+    off += (size_t)std::max<int32_t>(H.nlaunch, 1);
+  }
+  CUDA_TRY(cudaGetLastError());
+  CUDA_TRY(cudaMemcpyAsync(hv, bm, nb * sizeof(double), cudaMemcpyDeviceToHost, g->stream));
+  CUDA_TRY(cudaStreamSynchronize(g->stream));
+  const double* h = static_cast<const double*>(hv);
+  double total = 0.0;
+  off = 0;
+  for (int L = 0; L < g->levels; ++L) {
     double sL = 0.0;
-    for (double x : h) sL += x;
+    for (int32_t b = 0; b < g->host[L].nlaunch; ++b) sL += h[off + b];
+    off += (size_t)std::max<int32_t>(g->host[L].nlaunch, 1);
     total += sL * std::ldexp(1.0, -3 * L);
   }
   *mass = total;
@@ -1205,6 +1257,8 @@ void lbm_grid_destroy(lbm_grid* g) {
   for (int p = 0; p < 2; ++p)
     if (g->graph[p]) cudaGraphExecDestroy(g->graph[p]);
   for (auto& h : g->ipc_open) cudaIpcCloseMemHandle(h.second);
+  if (g->scratch) cudaFree(g->scratch);
+  if (g->hscratch) cudaFreeHost(g->hscratch);
   for (void* p : g->allocs) cudaFree(p);
   if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
   delete g;
