@@ -54,6 +54,7 @@ def _load():
         lib.ora_create.restype = P
         lib.ora_destroy.argtypes = [P]
         lib.ora_force_gamma2.argtypes = [P, ctypes.c_int]
+        lib.ora_set_variant.argtypes = [P, ctypes.c_int]
         lib.ora_num_leaves.argtypes = [P, ctypes.c_int]
         lib.ora_num_leaves.restype = ctypes.c_int64
         lib.ora_init_equilibrium.argtypes = [P, ctypes.c_int, dp, dp]
@@ -136,6 +137,10 @@ class Oracle:
         if h is not None and h.value:
             self.lib.ora_destroy(h)
             self.h = None
+
+    def set_variant(self, variant: str):
+        """"paper" (default) or "volumetric" (ghost advection)."""
+        self.lib.ora_set_variant(self.h, {"paper": 0, "volumetric": 1}[variant])
 
     def force_gamma2(self, on: bool = True):
         self.lib.ora_force_gamma2(self.h, int(on))
