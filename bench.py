@@ -182,6 +182,9 @@ def main():
     ap.add_argument("--config", default="tunnel4", choices=sorted(CONFIGS))
     ap.add_argument("--precision", default=None, choices=["fp32", "fp64"],
                     help="default fp32 (fp64 for the Tab. I sphere configs, the paper's precision)")
+    ap.add_argument("--variant", default="paper", choices=["paper", "volumetric"],
+                    help="interface transport: the paper's method (default) or the volumetric "
+                         "ghost-advection variant (DESIGN.md §16)")
     ap.add_argument("--schedule", default="fused", choices=sorted(SCHEDULES),
                     help="fusion ablation (lbm_set_schedule); the default is the product schedule")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -216,7 +219,8 @@ def main():
     t0 = time.perf_counter()
     # N > 1: rank's x-slab of the SAME workload (strong scaling), halos written
     # into the neighbour GPUs' buffers by the level kernels (CUDA IPC / NVLink)
-    g = lbmr.grid_from_problem(prob, precision=prec, stream=stream.cuda_stream, init=False, n_ranks=ws, rank=rank)
+    g = lbmr.grid_from_problem(prob, precision=prec, stream=stream.cuda_stream, init=False, n_ranks=ws, rank=rank,
+                               variant=lbmr.VARIANT_VOLUMETRIC if args.variant == "volumetric" else lbmr.VARIANT_PAPER)
     if ws > 1:
         import torch.distributed as dist
         blobs = {side: (g.halo_export(side) if lbmr.g_has(g, side) else None) for side in (0, 1)}
@@ -337,7 +341,8 @@ def main():
             "config": {"workload": desc, "levels": prob.levels, "leaves": leaves, "updates_per_step": upd,
                        "parallelism": f"x-slabs x{ws} (halo peer stores over NVLink)" if ws > 1 else "single",
                        "l2": f"working set {dev_bytes / 1e9:.2f} GB > 126 MB L2 (no flush needed)",
-                       "precision": args.precision, "schedule": args.schedule, "setup_s": round(setup_s, 2),
+                       "precision": args.precision, "schedule": args.schedule, "variant": args.variant,
+                       "setup_s": round(setup_s, 2),
                        **({"paper_a100_fp64_mlups": PAPER_MLUPS[args.config]} if args.config in PAPER_MLUPS else {})},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "kernel": f"level_step L{dom}",

@@ -69,7 +69,13 @@ typedef struct {
   double omega0;            /* level-0 relaxation Δt/τ; ω_L by Eq.9                 */
   int32_t n_ranks, rank;    /* x-slab partition; (1, 0) = whole domain on this device        */
   void* stream;             /* cudaStream_t to enqueue on; NULL = library-owned stream      */
+  int32_t variant;          /* LBM_VARIANT_PAPER (0): the paper's method as read in DESIGN.md
+                               §3 (default).  LBM_VARIANT_VOLUMETRIC (1): fine-ghost advection,
+                               mass-exact on interface edges/corners (single
+                               rank; LBM_E_UNSUPPORTED where a wall touches the coarse side of
+                               an interface in a way the traces cannot express)              */
 } lbm_grid_desc;
+enum { LBM_VARIANT_PAPER = 0, LBM_VARIANT_VOLUMETRIC = 1 };
 
 typedef struct lbm_grid lbm_grid;
 

@@ -60,6 +60,9 @@ struct DevLevel {
   uint32_t* ghost_fill = nullptr;
   uint32_t* coal_fill = nullptr;
   uint32_t* coal_cand = nullptr;
+  uint32_t* vfill = nullptr;   // volumetric variant lists (grid_builder.h)
+  uint32_t* vavg = nullptr;
+  void* vtemp = nullptr;
   void* pop[2] = {nullptr, nullptr};
   // neighbour rank on each side: its population buffers and the halo cell
   // index (in its grid) of every entry of our send list
@@ -200,6 +203,13 @@ StepParams<T> make_params(const lbm_grid* g, int L, int64_t k) {
   p.nfluid = g->host[L].nlaunch;
   p.ghost_fill = D.ghost_fill;
   p.nghost = (int32_t)(g->host[L].ghost_fill.size() / 2);
+  p.vtemp = static_cast<const T*>(D.vtemp);
+  if (g->desc.variant == LBM_VARIANT_VOLUMETRIC && L > 0 && ((k + 1) & 1) == 0) {
+    // next substep is the second of the parent's substep: advected ghost packets
+    p.nghost = 0;
+    p.vfill = D.vfill;
+    p.nvfill = (int32_t)(g->host[L].vfill.size() / 8);
+  }
   if (L > 0) p.gsrc = static_cast<const T*>(g->dev[L - 1].pop[((k + 2) / 2) & 1]);  // C_{L-1}^{ceil((k+1)/2)}
   if (g->n_ranks > 1) {
     const HostLevel& H = g->host[L];
@@ -225,8 +235,13 @@ void launch_F_typed(lbm_grid* g, int L, int64_t k, int kind) {
     launch_level_step(g->Q, g->coll, g->prec, 1, &p, g->stream);
     return;
   }
-  // coalescence ghosts of C_L^k from C_{L+1}^{2k-1} and C_{L+1}^{2k} (both ready now)
   const HostLevel& H = g->host[L];
+  // volumetric variant: coarse averages of the children's arrivals into the
+  // slots F_L^k pulls (gather, then scatter: DESIGN.md §16)
+  if (!H.vavg.empty())
+    launch_vavg(g->Q, g->prec, g->dev[L].vavg, (int32_t)(H.vavg.size() / 36), g->dev[L].pop[k & 1],
+                g->dev[L + 1].pop[1], g->dev[L + 1].pop[0], g->bc_dev, g->face_dev, g->dev[L].vtemp, g->stream);
+  // coalescence ghosts of C_L^k from C_{L+1}^{2k-1} and C_{L+1}^{2k} (both ready now)
   if (L + 1 < g->levels && !H.coal_fill.empty()) {
     if (g->n_ranks > 1) {
       // the gather reads L+1 halo cells: it follows the neighbour wait of F_L^k,
@@ -387,6 +402,9 @@ static lbm_status validate_desc(const lbm_grid_desc* d, int32_t levels, const ui
     }
   }
   if (d->n_ranks < 1 || d->rank < 0 || d->rank >= d->n_ranks) return fail(LBM_E_INVAL, "bad n_ranks / rank");
+  if (d->variant != LBM_VARIANT_PAPER && d->variant != LBM_VARIANT_VOLUMETRIC) return fail(LBM_E_INVAL, "bad variant");
+  if (d->variant == LBM_VARIANT_VOLUMETRIC && d->n_ranks > 1)
+    return fail(LBM_E_UNSUPPORTED, "the volumetric variant is single-rank only");
   if (d->n_ranks > d->nx) return fail(LBM_E_INVAL, "more ranks than level-0 x cells");
   for (int L = 0; L < levels; ++L) {
     int64_t n0 = (int64_t)d->nx << L, n1 = (int64_t)d->ny << L, n2 = (int64_t)d->nz << L;
@@ -470,6 +488,7 @@ static lbm_status build_host(const lbm_grid_desc* d, int32_t levels, const uint8
   in.levels = levels;
   in.Q = d->lattice;
   in.masks = masks;
+  in.variant = d->variant;
   if (slab) {
     in.n0[0] = slab->desc.nx;
     in.periodic[0] = 0;
@@ -498,6 +517,7 @@ static void fill_info(const std::vector<HostLevel>& host, int Q, int prec, lbm_g
   info->launches_per_step = info->kernels_per_step;
   for (size_t L = 0; L < host.size(); ++L) {
     if (!host[L].coal_fill.empty()) info->launches_per_step += (int64_t)1 << L;
+    if (!host[L].vavg.empty()) info->launches_per_step += (int64_t)2 << L;
     info->leaves[L] = host[L].leaves;
     info->blocks[L] = host[L].nfluid;
     info->special_blocks[L] = host[L].nspecial;
@@ -610,6 +630,9 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     if ((s = dev_upload(g, &D.ghost_fill, H.ghost_fill))) return cleanup(s);
     if ((s = dev_upload(g, &D.coal_fill, H.coal_fill))) return cleanup(s);
     if ((s = dev_upload(g, &D.coal_cand, H.coal_cand))) return cleanup(s);
+    if ((s = dev_upload(g, &D.vfill, H.vfill))) return cleanup(s);
+    if ((s = dev_upload(g, &D.vavg, H.vavg))) return cleanup(s);
+    if ((s = dev_alloc(g, &D.vtemp, (H.vavg.size() / 36) * g->tsize))) return cleanup(s);
     for (int b = 0; b < 2; ++b) {
       if ((s = dev_alloc(g, &D.pop[b], pop_bytes(g, L)))) return cleanup(s);
       if (cudaMemset(D.pop[b], 0, pop_bytes(g, L)) != cudaSuccess) return cleanup(fail(LBM_E_CUDA, "memset"));

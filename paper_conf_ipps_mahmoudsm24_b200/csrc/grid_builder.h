@@ -39,6 +39,11 @@ struct HostLevel {
   std::vector<uint32_t> ghost_fill;   // pairs {ghost cell at L, parent cell at L-1} (block*512+local)
   std::vector<uint32_t> coal_fill;    // pairs {dest population index (ghost, q), (|B|-1) << 26 | first candidate}
   std::vector<uint32_t> coal_cand;    // fine candidate population indices (level L+1)
+  // volumetric variant: expressions are uint4 {pop index,
+  // tag | nwall << 4 | wall0 << 8, wall1 | wall2 << 16, 0} (lattice.h kVt*)
+  std::vector<uint32_t> vfill;        // [n][8]: {dst pop index, 0, 0, 0, expr}: the second-substep ghost packets
+  std::vector<uint32_t> vavg;         // [n][36]: {slot pop index or ~0u, 0, 0, 0, 8 exprs}: coarse averages
+  std::vector<uint32_t> avg_base;     // host only: [nblocks*512] first vavg entry of an averaged cell, or ~0u
   std::vector<int32_t> plain_ids;     // fluid blocks without special cells (Morton order)
   std::vector<int32_t> special_ids;   // the others (Morton order)
 };
@@ -55,6 +60,7 @@ struct BuildInput {
   // neighbour (0: -x, 1: +x)
   int32_t owned_lo0 = 0, owned_hi0 = -1;
   int32_t has_nb[2] = {0, 0};
+  int32_t variant = 0;                // 0 paper's method, 1 volumetric ghost advection
 };
 
 // Returns 0 on success; otherwise an lbm_status code with `err` filled.

@@ -48,6 +48,12 @@ struct StepParams {
   const uint32_t* ghost_fill;   // pairs {ghost cell, parent cell}
   int32_t nghost;
   const T* gsrc;                // C_{L-1}^{ceil((k+1)/2)}
+  // volumetric variant: when the next substep is the second
+  // one of the parent's substep, the trailing CTAs evaluate these per-(ghost,
+  // q) expressions (8 words each) instead of copying parents (nghost = 0)
+  const uint32_t* vfill;
+  int32_t nvfill;
+  const T* vtemp;               // coarse averages of this level (kLinkTemp records)
   // ---- x-slab partition (multi-GPU); unused when nbctas == 0 -------------
   int32_t nbctas;               // CTAs taking part in the halo protocol (cut-plane blocks, >= 1)
   int32_t nboundary;            // cut-plane blocks (stored and launched first)
@@ -70,6 +76,12 @@ void launch_coalesce(int Q, int precision, const void* fa, const void* fb, void*
 // (-1 -> NaN), read from the post-collision buffer `pop`.
 void launch_probe(int Q, int precision, const void* pop, const int64_t* cell, int64_t n, double* rho, double* u,
                   cudaStream_t s);
+
+// Volumetric variant: coarse averages of level L before F_L^k.
+// ent: [n][36] {slot, 0, 0, 0, 8 expressions}; A = C_L^k, B = C_{L+1}^{2k-1},
+// C = C_{L+1}^{2k}; tmp[n] receives the means; then the slots are written.
+void launch_vavg(int Q, int precision, const uint32_t* ent, int32_t n, void* A, const void* B, const void* C,
+                 const BCEntry* bc, const uint8_t* face_cls, void* tmp, cudaStream_t s);
 
 // One-thread kernel: wait until both neighbours (has_nb) have completed the
 // cut-plane part of every kernel this rank has completed.

@@ -69,7 +69,15 @@ constexpr unsigned kNoBCSource = 0xffffffffu;
 //  kLinkBC     w0 = BC class of the source leaf
 //  kLinkFace   w0 = outside pattern (ox+1)+3(oy+1)+9(oz+1) -> class via face table
 //  kLinkCoal   w0 = first index in the coalescence list, w1 & 0xf = |B|
-constexpr unsigned kLinkSame = 0, kLinkCoarse = 1, kLinkBC = 2, kLinkFace = 3, kLinkCoal = 4;
+//  kLinkTemp   w0 = index into the level's volumetric averages
+constexpr unsigned kLinkSame = 0, kLinkCoarse = 1, kLinkBC = 2, kLinkFace = 3, kLinkCoal = 4, kLinkTemp = 5;
+
+// volumetric-variant expression tags (which buffer the population index is in)
+//  fill list of level L (run by F_L^{k-1}):  kVtA = C_L^{k-1}, kVtB = C_{L-1}
+//  average list of level L (before F_L^k):   kVtA = C_L^k, kVtB = C_{L+1}^{2k-1}, kVtC = C_{L+1}^{2k}
+// walls: 14 bits each, BC source (class < 256 or kFaceSourceBase + pattern)
+// | direction << 9, applied innermost first
+constexpr unsigned kVtNone = 0, kVtA = 1, kVtB = 2, kVtC = 3;
 
 // cell type codes stored per block (mask codes + derived states)
 constexpr unsigned char kAbsent = 0;    // covered by a coarser leaf, or outside the domain

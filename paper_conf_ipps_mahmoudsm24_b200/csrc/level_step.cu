@@ -307,8 +307,9 @@ __device__ __forceinline__ void resolve_slow_sv(const StepParams<T>& P, T* sv, u
       v[b] = T(0);
       if (qb[b] >= 0) {
         const unsigned tag = eb[b].y >> 28;
-        const T* base = (tag == kLinkCoarse) ? P.csrc : P.src;
-        const unsigned idx = (tag <= kLinkCoarse) ? eb[b].x : own + (unsigned)(opp_rt(qb[b]) * kCells);
+        const T* base = (tag == kLinkCoarse) ? P.csrc : (tag == kLinkTemp ? P.vtemp : P.src);
+        const unsigned idx =
+            (tag <= kLinkCoarse || tag == kLinkTemp) ? eb[b].x : own + (unsigned)(opp_rt(qb[b]) * kCells);
         v[b] = __ldg(base + idx);
       }
     }
@@ -535,6 +536,48 @@ __device__ __forceinline__ void ghost_fill_one(const StepParams<T>& P, int i) {
 
 __host__ __device__ constexpr int ghost_ctas(int n) { return (n + 255) / 256; }
 
+// Volumetric variant: one gather expression = a population of
+// buffer A, B or C (tag) followed by up to three wall reflections, innermost
+// first (halfway bounce-back as the oracle's wall_value: NOSLIP keeps the
+// value, VELOCITY adds 6 w_d e_d.u_w, OUTFLOW gives f = w, i.e. g = 0).
+template <int Q, typename T>
+__device__ __forceinline__ T vexpr(const uint32_t* e, const T* A, const T* B, const T* C, const BCEntry* bc,
+                                   const uint8_t* face_cls) {
+  const uint32_t tag = e[1] & 15u, nw = (e[1] >> 4) & 3u;
+  T v = T(0);
+  if (tag == kVtA) v = A[e[0]];
+  else if (tag == kVtB) v = B[e[0]];
+  else if (tag == kVtC) v = C[e[0]];
+  for (uint32_t w = 0; w < nw; ++w) {
+    const uint32_t wd = w == 0 ? (e[1] >> 8) & 0x3fffu : (w == 1 ? e[2] & 0xffffu : e[2] >> 16);
+    const uint32_t src = wd & 511u, dir = wd >> 9;
+    const unsigned cls = src < kFaceSourceBase ? src : (unsigned)__ldg(face_cls + (src - kFaceSourceBase));
+    const int kind = __ldg(&bc[cls].kind);
+    if (kind == LBM_BC_OUTFLOW) {
+      v = T(0);
+    } else if (kind == LBM_BC_VELOCITY) {
+      const double eu = c_ex[dir] * __ldg(&bc[cls].u[0]) + c_ey[dir] * __ldg(&bc[cls].u[1]) +
+                        c_ez[dir] * __ldg(&bc[cls].u[2]);
+      v += T(6.0 * wq_rt<Q>(dir) * 1.0 * eu);
+    }
+  }
+  return v;
+}
+
+// Trailing CTAs of a level kernel: refresh the ghosts the next kernel of this
+// level pulls — parent copies (Eq.10), or in the volumetric variant's second
+// substep the advected packets.
+template <int Q, typename T>
+__device__ __forceinline__ void trail_fill(const StepParams<T>& P, int i) {
+  ghost_fill_one<Q, T>(P, i);
+  if (i < P.nvfill) {
+    const uint32_t* e = P.vfill + 8 * (size_t)i;
+    P.dst[e[0]] = vexpr<Q, T>(e + 4, P.src, P.gsrc, nullptr, P.bc, P.face_cls);
+  }
+}
+
+__host__ __device__ inline int trail_items(int nghost, int nvfill) { return nghost > nvfill ? nghost : nvfill; }
+
 // Minimum resident CTAs per SM (register budget 65536 / (256 * MINB)),
 // chosen per variant from ptxas -v and measurement.
 #ifndef LBMR_OCC_Q19F
@@ -687,7 +730,7 @@ __global__ void __launch_bounds__(kStepThreads, (PlainOcc<Q, T, COLL>::value * 2
     level_step_all(const StepParams<T> P) {
   const int main = P.nfluid * 512 / kStepThreads;
   if ((int)blockIdx.x >= main) {  // trailing CTAs refresh the explosion ghosts
-    ghost_fill_one<Q, T>(P, ((int)blockIdx.x - main) * kStepThreads + threadIdx.x);
+    trail_fill<Q, T>(P, ((int)blockIdx.x - main) * kStepThreads + threadIdx.x);
     return;
   }
   if (kStepThreads == 512) step_cell<Q, COLL, T, false>(P, blockIdx.x, threadIdx.x);
@@ -719,18 +762,18 @@ __global__ void __launch_bounds__(256, PlainOcc<Q, T, COLL>::value) level_step_h
   const bool fill = (int)blockIdx.x >= main;
   const bool proto = (int)blockIdx.x < P.nbctas || fill;
   if (fill) {
-    ghost_fill_one<Q, T>(P, ((int)blockIdx.x - main) * 256 + threadIdx.x);
+    trail_fill<Q, T>(P, ((int)blockIdx.x - main) * 256 + threadIdx.x);
   } else if (blk < P.nfluid) {
     if (STREAM) step_cell<Q, COLL, T, true>(P, blk, t);
     else collide_cell<Q, COLL, T, true>(P, blk, t);
   }
-  if (proto) halo_signal<T>(P, P.nbctas + ghost_ctas(P.nghost));
+  if (proto) halo_signal<T>(P, P.nbctas + ghost_ctas(trail_items(P.nghost, P.nvfill)));
 }
 
 template <int Q, int COLL, typename T>
 __global__ void __launch_bounds__(256) level_collide(const StepParams<T> P) {
   if ((int)blockIdx.x >= 2 * P.nfluid) {
-    ghost_fill_one<Q, T>(P, ((int)blockIdx.x - 2 * P.nfluid) * 256 + threadIdx.x);
+    trail_fill<Q, T>(P, ((int)blockIdx.x - 2 * P.nfluid) * 256 + threadIdx.x);
     return;
   }
   collide_cell<Q, COLL, T, false>(P, blockIdx.x >> 1, ((blockIdx.x & 1) << 8) | threadIdx.x);
@@ -745,7 +788,7 @@ template <int Q, typename T>
 __global__ void __launch_bounds__(256, PlainOcc<Q, T, LBM_BGK>::value) level_stream(const StepParams<T> P) {
   const int main = 2 * P.nfluid;
   if ((int)blockIdx.x >= main) {
-    ghost_fill_one<Q, T>(P, ((int)blockIdx.x - main) * 256 + threadIdx.x);
+    trail_fill<Q, T>(P, ((int)blockIdx.x - main) * 256 + threadIdx.x);
     return;
   }
   step_cell<Q, LBM_BGK, T, false, false>(P, blockIdx.x >> 1, ((blockIdx.x & 1) << 8) | threadIdx.x);
@@ -879,6 +922,46 @@ __global__ void __launch_bounds__(256) coalesce_kernel(const T* __restrict__ fa,
   dst[d] = acc / T(2 * cnt);
 }
 
+template <int Q, typename T>
+__global__ void __launch_bounds__(256) vavg_gather(const uint32_t* __restrict__ ent, int n, const T* A, const T* B,
+                                                   const T* C, const BCEntry* bc, const uint8_t* face_cls, T* tmp) {
+  const int i = blockIdx.x * 256 + threadIdx.x;
+  if (i >= n) return;
+  const uint32_t* e = ent + 36 * (size_t)i;
+  T acc = T(0);
+#pragma unroll
+  for (int m = 0; m < 8; ++m) acc += vexpr<Q, T>(e + 4 + 4 * m, A, B, C, bc, face_cls);
+  tmp[i] = acc / T(8);
+}
+
+template <typename T>
+__global__ void __launch_bounds__(256) vavg_scatter(const uint32_t* __restrict__ ent, int n, const T* tmp, T* A) {
+  const int i = blockIdx.x * 256 + threadIdx.x;
+  if (i >= n) return;
+  const uint32_t slot = __ldg(ent + 36 * (size_t)i);
+  if (slot != ~0u) A[slot] = tmp[i];
+}
+
+template <int Q, typename T>
+static void vavg_typed(const uint32_t* ent, int32_t n, void* A, const void* B, const void* C, const BCEntry* bc,
+                       const uint8_t* fc, void* tmp, cudaStream_t s) {
+  const int grid = (n + 255) / 256;
+  vavg_gather<Q, T><<<grid, 256, 0, s>>>(ent, n, (const T*)A, (const T*)B, (const T*)C, bc, fc, (T*)tmp);
+  vavg_scatter<T><<<grid, 256, 0, s>>>(ent, n, (const T*)tmp, (T*)A);
+}
+
+void launch_vavg(int Q, int precision, const uint32_t* ent, int32_t n, void* A, const void* B, const void* C,
+                 const BCEntry* bc, const uint8_t* face_cls, void* tmp, cudaStream_t s) {
+  if (n <= 0) return;
+  if (precision == LBM_FP32) {
+    if (Q == 19) vavg_typed<19, float>(ent, n, A, B, C, bc, face_cls, tmp, s);
+    else vavg_typed<27, float>(ent, n, A, B, C, bc, face_cls, tmp, s);
+  } else {
+    if (Q == 19) vavg_typed<19, double>(ent, n, A, B, C, bc, face_cls, tmp, s);
+    else vavg_typed<27, double>(ent, n, A, B, C, bc, face_cls, tmp, s);
+  }
+}
+
 void launch_halo_wait(const unsigned long long* flags, int nb0, int nb1, cudaStream_t s) {
   halo_wait_kernel<<<1, 1, 0, s>>>(flags, nb0, nb1);
 }
@@ -905,7 +988,7 @@ static void launch_typed(int kind, const void* params, cudaStream_t s) {
   const StepParams<T>& p = *static_cast<const StepParams<T>*>(params);
   dim3 block(256);
   const size_t sm = slow_smem<Q, T>();
-  const int gc = ghost_ctas(p.nghost);
+  const int gc = ghost_ctas(trail_items(p.nghost, p.nvfill));
   if (p.nbctas > 0) {  // partitioned: always launched (the protocol must run)
     halo_wait_kernel<<<1, 1, 0, s>>>(p.flags, p.has_nb[0], p.has_nb[1]);
     dim3 grid(2 * std::max(p.nfluid, 1) + gc);
@@ -913,7 +996,7 @@ static void launch_typed(int kind, const void* params, cudaStream_t s) {
     else level_step_halo<Q, COLL, T, true><<<grid, block, sm, s>>>(p);
     return;
   }
-  if (p.nfluid <= 0 && p.nghost <= 0) return;
+  if (p.nfluid <= 0 && p.nghost <= 0 && p.nvfill <= 0) return;
   if (kind == 1) {
     level_collide<Q, COLL, T><<<dim3(2 * p.nfluid + gc), block, 0, s>>>(p);
   } else if (kind == 3) {
@@ -921,7 +1004,7 @@ static void launch_typed(int kind, const void* params, cudaStream_t s) {
   } else if (kind == 4) {
     if (p.nfluid > 0) level_collide_inplace<Q, COLL, T><<<dim3(2 * p.nfluid), block, 0, s>>>(p);
   } else {
-    const int gct = (p.nghost + kStepThreads - 1) / kStepThreads;
+    const int gct = (trail_items(p.nghost, p.nvfill) + kStepThreads - 1) / kStepThreads;
     level_step_all<Q, COLL, T><<<dim3(p.nfluid * 512 / kStepThreads + gct), dim3(kStepThreads), sm, s>>>(p);
   }
 }
@@ -957,6 +1040,12 @@ void preload_kernels() {
   cudaFuncGetAttributes(&a, halo_wait_kernel);
   cudaFuncGetAttributes(&a, coalesce_kernel<float>);
   cudaFuncGetAttributes(&a, probe_kernel<19, float>);
+  cudaFuncGetAttributes(&a, vavg_gather<19, float>);
+  cudaFuncGetAttributes(&a, vavg_gather<27, float>);
+  cudaFuncGetAttributes(&a, vavg_gather<19, double>);
+  cudaFuncGetAttributes(&a, vavg_gather<27, double>);
+  cudaFuncGetAttributes(&a, vavg_scatter<float>);
+  cudaFuncGetAttributes(&a, vavg_scatter<double>);
   cudaFuncGetAttributes(&a, probe_kernel<27, float>);
   cudaFuncGetAttributes(&a, probe_kernel<19, double>);
   cudaFuncGetAttributes(&a, probe_kernel<27, double>);

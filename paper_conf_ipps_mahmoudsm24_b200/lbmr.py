@@ -23,6 +23,7 @@ BGK, KBC = 0, 1
 FP32, FP64 = 0, 1
 BC_NOSLIP, BC_VELOCITY, BC_OUTFLOW = 0, 1, 2
 SCHED_FUSED, SCHED_UNFUSED, SCHED_NO_GRAPH = 0, 1, 2
+VARIANT_PAPER, VARIANT_VOLUMETRIC = 0, 1
 
 
 class LBMError(RuntimeError):
@@ -40,6 +41,7 @@ class GridDesc(ctypes.Structure):
         ("omega0", ctypes.c_double),
         ("n_ranks", ctypes.c_int32), ("rank", ctypes.c_int32),
         ("stream", ctypes.c_void_p),
+        ("variant", ctypes.c_int32),
     ]
 
 
@@ -133,7 +135,7 @@ def _dp(a: Optional[np.ndarray]):
 
 
 def make_desc(nx, ny, nz, periodic=(0, 0, 0), face_bc=(0,) * 6, lattice=D3Q19, collision=BGK, precision=FP32,
-              omega0=1.0, stream=None, n_ranks=1, rank=0) -> GridDesc:
+              omega0=1.0, stream=None, n_ranks=1, rank=0, variant=VARIANT_PAPER) -> GridDesc:
     d = GridDesc()
     d.nx, d.ny, d.nz = nx, ny, nz
     for a in range(3):
@@ -144,6 +146,7 @@ def make_desc(nx, ny, nz, periodic=(0, 0, 0), face_bc=(0,) * 6, lattice=D3Q19, c
     d.omega0 = float(omega0)
     d.n_ranks, d.rank = int(n_ranks), int(rank)
     d.stream = stream
+    d.variant = int(variant)
     return d
 
 
@@ -233,7 +236,7 @@ class Grid:
     def __init__(self, nx: int, ny: int, nz: int, masks: Sequence[np.ndarray], *, periodic=(0, 0, 0),
                  face_bc=(0, 0, 0, 0, 0, 0), lattice: int = D3Q19, collision: int = BGK,
                  precision: int = FP32, omega0: float = 1.0, stream: Optional[int] = None,
-                 n_ranks: int = 1, rank: int = 0):
+                 n_ranks: int = 1, rank: int = 0, variant: int = VARIANT_PAPER):
         lib = load_library()
         self.lib = lib
         self.shape0 = (nx, ny, nz)
@@ -242,7 +245,8 @@ class Grid:
         for L, m in enumerate(self._masks):
             if m.shape != (nx << L, ny << L, nz << L):
                 raise ValueError(f"mask {L} has shape {m.shape}, expected {(nx << L, ny << L, nz << L)}")
-        d = make_desc(nx, ny, nz, periodic, face_bc, lattice, collision, precision, omega0, stream, n_ranks, rank)
+        d = make_desc(nx, ny, nz, periodic, face_bc, lattice, collision, precision, omega0, stream, n_ranks, rank,
+                      variant)
         self.n_ranks, self.rank = n_ranks, rank
         self._periodic_x = bool(periodic[0])
         ptrs = (ctypes.c_void_p * self.levels)(*[m.ctypes.data for m in self._masks])
@@ -375,11 +379,11 @@ class Grid:
 
 
 def grid_from_problem(prob, precision: int = FP32, stream: Optional[int] = None, init: bool = True,
-                      n_ranks: int = 1, rank: int = 0) -> Grid:
+                      n_ranks: int = 1, rank: int = 0, variant: int = VARIANT_PAPER) -> Grid:
     """Build a Grid from an ``lbm_inputs.Problem`` (masks, BCs, initial state);
     with n_ranks > 1 the grid holds rank's x-slab (connect its halos before
     stepping)."""
-    g = Grid(prob.nx, prob.ny, prob.nz, prob.masks, stream=stream, n_ranks=n_ranks, rank=rank,
+    g = Grid(prob.nx, prob.ny, prob.nz, prob.masks, stream=stream, n_ranks=n_ranks, rank=rank, variant=variant,
              **_problem_kw(prob, precision))
     for cls, (kind, u) in prob.bc.items():
         g.set_bc(cls, kind, u)
