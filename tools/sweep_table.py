@@ -8,7 +8,8 @@ for f in sorted(sys.argv[1:]):
         print(f"{f}: no bench line")
         continue
     c = d["config"]
-    rows.append((c["workload"].split(":")[0], c.get("precision"), c.get("schedule", "fused"), d["value"],
+    rows.append((c["workload"].split(":")[0], c.get("precision"),
+                 c.get("schedule", "fused") + ("/vol" if c.get("variant") == "volumetric" else ""), d["value"],
                  d["roofline"]["frac"], [round(p["GBs"]) for p in d["per_level"]], d.get("vs_baseline"),
                  d["clocks"].get("sm_mhz")))
 for r in rows:
