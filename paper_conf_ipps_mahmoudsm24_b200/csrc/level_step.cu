@@ -569,6 +569,9 @@ __device__ __forceinline__ T vexpr(const uint32_t* e, const T* A, const T* B, co
 // substep the advected packets.
 template <int Q, typename T>
 __device__ __forceinline__ void trail_fill(const StepParams<T>& P, int i) {
+#ifdef LBMR_DEBUG_NOFILL
+  return;  // timing experiment only (wrong results)
+#endif
   ghost_fill_one<Q, T>(P, i);
   if (i < P.nvfill) {
     const uint32_t* e = P.vfill + 8 * (size_t)i;
