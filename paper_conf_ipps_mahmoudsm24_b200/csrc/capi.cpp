@@ -202,7 +202,7 @@ StepParams<T> make_params(const lbm_grid* g, int L, int64_t k) {
   p.face_cls = g->face_dev;
   p.nfluid = g->host[L].nlaunch;
   p.ghost_fill = D.ghost_fill;
-  p.nghost = (int32_t)(g->host[L].ghost_fill.size() / 2);
+  p.nghost = (int32_t)(g->host[L].ghost_fill.size() / 3);
   p.vtemp = static_cast<const T*>(D.vtemp);
   if (g->desc.variant == LBM_VARIANT_VOLUMETRIC && L > 0 && ((k + 1) & 1) == 0) {
     // next substep is the second of the parent's substep: advected ghost packets

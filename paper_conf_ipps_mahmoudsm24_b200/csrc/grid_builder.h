@@ -36,7 +36,7 @@ struct HostLevel {
   // explosion ghosts (ABSENT cells pulled by fluid leaves, parent a fluid
   // leaf at L-1): stored, refreshed by the level's previous kernel
   std::vector<uint8_t> ghost;         // [nblocks*512] host only: 1 explosion ghost, 2 coalescence ghost
-  std::vector<uint32_t> ghost_fill;   // pairs {ghost cell at L, parent cell at L-1} (block*512+local)
+  std::vector<uint32_t> ghost_fill;   // triples {ghost cell at L, parent cell at L-1 (block*512+local), pulled-q mask}
   std::vector<uint32_t> coal_fill;    // pairs {dest population index (ghost, q), (|B|-1) << 26 | first candidate}
   std::vector<uint32_t> coal_cand;    // fine candidate population indices (level L+1)
   // volumetric variant: expressions are uint4 {pop index,

@@ -45,7 +45,7 @@ struct StepParams {
   int32_t nfluid;               // blocks launched (owned fluid blocks, cut-plane blocks first)
   // explosion ghosts of the destination buffer, refreshed from the coarse
   // post-collision state the NEXT kernel of this level reads (Eq.10)
-  const uint32_t* ghost_fill;   // pairs {ghost cell, parent cell}
+  const uint32_t* ghost_fill;   // triples {ghost cell, parent cell, mask of the pulled directions}
   int32_t nghost;
   const T* gsrc;                // C_{L-1}^{ceil((k+1)/2)}
   // volumetric variant: when the next substep is the second

@@ -523,15 +523,18 @@ __device__ __forceinline__ void store_cell(const T (&g)[Q], T* __restrict__ dst,
 
 // Explosion ghosts: ghost cell g of level L holds its parent's
 // C_{L-1} populations, so interface cells pull the exploded value (Eq.10)
-// as a plain same-level load.  One thread per ghost, all Q planes.
+// as a plain same-level load.  One thread per ghost; only the planes an owned
+// fluid leaf pulls are refreshed (5 of 19 on a flat D3Q19 interface).
 template <int Q, typename T>
 __device__ __forceinline__ void ghost_fill_one(const StepParams<T>& P, int i) {
   if (i >= P.nghost) return;
-  const uint32_t gc = __ldg(P.ghost_fill + 2 * i), pc = __ldg(P.ghost_fill + 2 * i + 1);
+  const uint32_t gc = __ldg(P.ghost_fill + 3 * i), pc = __ldg(P.ghost_fill + 3 * i + 1);
+  const uint32_t mask = __ldg(P.ghost_fill + 3 * i + 2);
   T* d = P.dst + (gc >> 9) * (unsigned)(Q * kCells) + (gc & 511u);
   const T* s = P.gsrc + (pc >> 9) * (unsigned)(Q * kCells) + (pc & 511u);
 #pragma unroll
-  for (int q = 0; q < Q; ++q) d[q * kCells] = __ldg(s + q * kCells);
+  for (int q = 1; q < Q; ++q)
+    if ((mask >> q) & 1u) d[q * kCells] = __ldg(s + q * kCells);
 }
 
 __host__ __device__ constexpr int ghost_ctas(int n) { return (n + 255) / 256; }
@@ -728,16 +731,30 @@ __device__ __forceinline__ void collide_cell(const StepParams<T>& P, int blk, in
 #endif
 constexpr int kStepThreads = LBMR_CTA512 ? 512 : 256;
 
+#ifndef LBMR_FILL_FIRST
+#define LBMR_FILL_FIRST 0
+#endif
 template <int Q, int COLL, typename T>
 __global__ void __launch_bounds__(kStepThreads, (PlainOcc<Q, T, COLL>::value * 256) / kStepThreads)
     level_step_all(const StepParams<T> P) {
+#if LBMR_FILL_FIRST
+  // leading CTAs refresh the explosion ghosts (they overlap the first wave)
+  const int lead = (trail_items(P.nghost, P.nvfill) + kStepThreads - 1) / kStepThreads;
+  if ((int)blockIdx.x < lead) {
+    trail_fill<Q, T>(P, (int)blockIdx.x * kStepThreads + threadIdx.x);
+    return;
+  }
+  const int b = (int)blockIdx.x - lead;
+#else
   const int main = P.nfluid * 512 / kStepThreads;
   if ((int)blockIdx.x >= main) {  // trailing CTAs refresh the explosion ghosts
     trail_fill<Q, T>(P, ((int)blockIdx.x - main) * kStepThreads + threadIdx.x);
     return;
   }
-  if (kStepThreads == 512) step_cell<Q, COLL, T, false>(P, blockIdx.x, threadIdx.x);
-  else step_cell<Q, COLL, T, false>(P, blockIdx.x >> 1, ((blockIdx.x & 1) << 8) | threadIdx.x);
+  const int b = (int)blockIdx.x;
+#endif
+  if (kStepThreads == 512) step_cell<Q, COLL, T, false>(P, b, threadIdx.x);
+  else step_cell<Q, COLL, T, false>(P, b >> 1, ((b & 1) << 8) | threadIdx.x);
 }
 
 // Partitioned variant: grid = 2 * max(nfluid, 1) CTAs; the first nbctas run
