@@ -249,7 +249,7 @@ void launch_F_typed(lbm_grid* g, int L, int64_t k, int kind) {
       launch_halo_wait(p.flags, p.has_nb[0], p.has_nb[1], g->stream);
     }
     launch_coalesce(g->Q, g->prec, g->dev[L + 1].pop[1], g->dev[L + 1].pop[0], g->dev[L].pop[k & 1],
-                    g->dev[L].coal_fill, g->dev[L].coal_cand, (int32_t)(H.coal_fill.size() / 2), g->stream);
+                    g->dev[L].coal_fill, g->dev[L].coal_cand, H.coal_n[0], H.coal_n[1], g->stream);
   }
   if (g->sched & LBM_SCHED_UNFUSED) {  // S_L^k then C_L^{k+1} in place (fusion ablation)
     launch_level_step(g->Q, g->coll, g->prec, 3, &p, g->stream);

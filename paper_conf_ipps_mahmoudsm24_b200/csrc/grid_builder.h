@@ -37,8 +37,10 @@ struct HostLevel {
   // leaf at L-1): stored, refreshed by the level's previous kernel
   std::vector<uint8_t> ghost;         // [nblocks*512] host only: 1 explosion ghost, 2 coalescence ghost
   std::vector<uint32_t> ghost_fill;   // triples {ghost cell at L, parent cell at L-1 (block*512+local), pulled-q mask}
-  std::vector<uint32_t> coal_fill;    // pairs {dest population index (ghost, q), (|B|-1) << 26 | first candidate}
-  std::vector<uint32_t> coal_cand;    // fine candidate population indices (level L+1)
+  std::vector<uint32_t> coal_fill;    // [n] dest population index (ghost, q), sorted by (q, dest) per segment
+  std::vector<uint32_t> coal_cand;    // SoA fine candidate population indices (level L+1), ~0u = empty:
+                                      // [kCoalSlots][coal_n[0]] then [kCoalSlotsMax][coal_n[1]]
+  int64_t coal_n[2] = {0, 0};         // entries with |B| <= kCoalSlots, and the others
   // volumetric variant: expressions are uint4 {pop index,
   // tag | nwall << 4 | wall0 << 8, wall1 | wall2 << 16, 0} (lattice.h kVt*)
   std::vector<uint32_t> vfill;        // [n][8]: {dst pop index, 0, 0, 0, expr}: the second-substep ghost packets

@@ -66,11 +66,12 @@ struct StepParams {
 };
 
 // Coalescence gather (Eq.11) into the coarse ghosts of `dst` (= C_L^k's
-// buffer, read next by F_L^k): for entry i, dst[fill[2i]] = (sum_B fa + sum_B fb)
-// / (2|B|) over the candidates cand[(fill[2i+1] & 0x3ffffff) ...], |B| =
-// (fill[2i+1] >> 26) + 1.
+// buffer, read next by F_L^k): for entry i, dst[fill[i]] = (sum_B fa + sum_B fb)
+// / (2|B|) over the filled candidate slots of entry i (grid_builder.h
+// coal_cand: n_main entries with kCoalSlots slots, then n_ovf entries with
+// kCoalSlotsMax slots, structure-of-arrays).
 void launch_coalesce(int Q, int precision, const void* fa, const void* fb, void* dst, const uint32_t* fill,
-                     const uint32_t* cand, int32_t n, cudaStream_t s);
+                     const uint32_t* cand, int64_t n_main, int64_t n_ovf, cudaStream_t s);
 
 // rho / u (double) of n cells given by population cell index block*512+local
 // (-1 -> NaN), read from the post-collision buffer `pop`.

@@ -79,6 +79,11 @@ constexpr unsigned kLinkSame = 0, kLinkCoarse = 1, kLinkBC = 2, kLinkFace = 3, k
 // | direction << 9, applied innermost first
 constexpr unsigned kVtNone = 0, kVtA = 1, kVtB = 2, kVtC = 3;
 
+// coalescence gather (Eq.11): candidate slots per entry.  |B| <= 4 on every
+// link of a planar interface; at most 7 of the 8 candidates 2p - e_q + c lie
+// outside the coarse leaf p (the one inside is ABSENT), so 7 bounds |B|.
+constexpr uint32_t kCoalSlots = 4, kCoalSlotsMax = 7;
+
 // cell type codes stored per block (mask codes + derived states)
 constexpr unsigned char kAbsent = 0;    // covered by a coarser leaf, or outside the domain
 constexpr unsigned char kFluid = 1;

@@ -924,22 +924,39 @@ void launch_probe(int Q, int precision, const void* pop, const int64_t* cell, in
   }
 }
 
-// Coalescence ghosts: one thread per (ghost cell, q) entry.
+// Coalescence ghosts: one thread per (ghost cell, q) entry,
+// entries ordered by (q, ghost) so a warp reads neighbouring fine cells of one
+// plane; candidate slots structure-of-arrays (grid_builder.h coal_cand).
 // Fine candidates summed in candidate order, first substep then second, like
 // the oracle (Eq.11, n = 2|B|, R-A2/R-A3).
+template <typename T, int K>
+__device__ __forceinline__ void coalesce_one(const T* __restrict__ fa, const T* __restrict__ fb, T* __restrict__ dst,
+                                             uint32_t d, const uint32_t* __restrict__ cand, int64_t stride) {
+  uint32_t c[K];
+#pragma unroll
+  for (int m = 0; m < K; ++m) c[m] = __ldg(cand + m * stride);
+  T acc = T(0);
+  unsigned cnt = 0;
+#pragma unroll
+  for (int m = 0; m < K; ++m)
+    if (c[m] != ~0u) { acc += __ldg(fa + c[m]); ++cnt; }
+#pragma unroll
+  for (int m = 0; m < K; ++m)
+    if (c[m] != ~0u) acc += __ldg(fb + c[m]);
+  dst[d] = acc / T(2 * cnt);
+}
+
 template <typename T>
 __global__ void __launch_bounds__(256) coalesce_kernel(const T* __restrict__ fa, const T* __restrict__ fb,
                                                        T* __restrict__ dst, const uint32_t* __restrict__ fill,
-                                                       const uint32_t* __restrict__ cand, int n) {
-  const int i = blockIdx.x * 256 + threadIdx.x;
-  if (i >= n) return;
-  const uint32_t d = __ldg(fill + 2 * i), w = __ldg(fill + 2 * i + 1);
-  const unsigned cnt = (w >> 26) + 1u;
-  const uint32_t* c = cand + (w & 0x3ffffffu);
-  T acc = T(0);
-  for (unsigned m = 0; m < cnt; ++m) acc += __ldg(fa + __ldg(c + m));
-  for (unsigned m = 0; m < cnt; ++m) acc += __ldg(fb + __ldg(c + m));
-  dst[d] = acc / T(2 * cnt);
+                                                       const uint32_t* __restrict__ cand, int64_t nmain, int64_t novf) {
+  const int64_t i = (int64_t)blockIdx.x * 256 + threadIdx.x;
+  if (i < nmain) {
+    coalesce_one<T, kCoalSlots>(fa, fb, dst, __ldg(fill + i), cand + i, nmain);
+  } else if (i < nmain + novf) {
+    const int64_t j = i - nmain;
+    coalesce_one<T, kCoalSlotsMax>(fa, fb, dst, __ldg(fill + i), cand + kCoalSlots * nmain + j, novf);
+  }
 }
 
 template <int Q, typename T>
@@ -987,14 +1004,17 @@ void launch_halo_wait(const unsigned long long* flags, int nb0, int nb1, cudaStr
 }
 
 void launch_coalesce(int Q, int precision, const void* fa, const void* fb, void* dst, const uint32_t* fill,
-                     const uint32_t* cand, int32_t n, cudaStream_t s) {
+                     const uint32_t* cand, int64_t n_main, int64_t n_ovf, cudaStream_t s) {
   (void)Q;
+  const int64_t n = n_main + n_ovf;
   if (n <= 0) return;
-  const int grid = (n + 255) / 256;
+  const unsigned grid = (unsigned)((n + 255) / 256);
   if (precision == LBM_FP32)
-    coalesce_kernel<float><<<grid, 256, 0, s>>>((const float*)fa, (const float*)fb, (float*)dst, fill, cand, n);
+    coalesce_kernel<float><<<grid, 256, 0, s>>>((const float*)fa, (const float*)fb, (float*)dst, fill, cand, n_main,
+                                                 n_ovf);
   else
-    coalesce_kernel<double><<<grid, 256, 0, s>>>((const double*)fa, (const double*)fb, (double*)dst, fill, cand, n);
+    coalesce_kernel<double><<<grid, 256, 0, s>>>((const double*)fa, (const double*)fb, (double*)dst, fill, cand,
+                                                  n_main, n_ovf);
 }
 
 // ---------------------------------------------------------------- dispatch
