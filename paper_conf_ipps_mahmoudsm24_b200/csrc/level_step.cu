@@ -128,22 +128,13 @@ __device__ __forceinline__ void collide_bgk(T (&g)[Q], T omega) {
   }
 }
 
-// KBC (reading R-A9) on shifted populations; D3Q27 only.
-//   f^neq = g - g^eq;  Δs from the deviatoric second moments of f^neq;
-//   Δh = f^neq - Δs;  γ = 1/β - (2 - 1/β) <Δs|Δh>/<Δh|Δh>,  <X|Y> = Σ X Y / f^eq;
-//   f* = f - β (2 Δs + γ Δh),  β = ω/2.
-// Organised for the ALU: g^eq by opposite pairs (shared even part), second
-// moments from pair sums (e_a e_b is even), one rounded reciprocal per f^eq.
 template <>
 __device__ __forceinline__ double recip<double>(double x) {
   return __drcp_rn(x);
 }
 
-// Register-lean form: g^eq is never stored.  It is recomputed from (δρ, j)
-// in each of the three passes that need it (f^neq, the entropic products,
-// the update); opaque copies of the moments (fresh()) stop the compiler from
-// merging the passes' recomputations back into 27 live registers, so the
-// live set is the 27 f^neq plus a few scalars (occupancy).
+// Opaque copy: stops the compiler from merging recomputations of g^eq in
+// separate passes back into values held live across them (occupancy).
 template <typename T>
 __device__ __forceinline__ T fresh(T x) {
   if constexpr (sizeof(T) == 4) asm volatile("" : "+f"(x));
@@ -151,23 +142,65 @@ __device__ __forceinline__ T fresh(T x) {
   return x;
 }
 
+// Reciprocal of a positive, normal f^eq_i inside the entropic products:
+// fp32 uses the one-instruction MUFU approximation (rel. error <= 2^-23, far
+// inside the fp32 parity bar); fp64 keeps the correctly rounded one.
+template <typename T>
+__device__ __forceinline__ T rcp_feq(T x) {
+  if constexpr (sizeof(T) == 4) {
+    float r;
+    asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+    return r;
+  } else {
+    return __drcp_rn(x);
+  }
+}
+
+// KBC (reading R-A9) on shifted populations; D3Q27 only:
+//   f^neq = g - g^eq;  Δs from the deviatoric second moments of f^neq;
+//   Δh = f^neq - Δs;  γ = 1/β - (2 - 1/β) <Δs|Δh>/<Δh|Δh>,  <X|Y> = Σ X Y / f^eq
+//   (γ = 2 if <Δh|Δh> < 1e-30);  f* = f - β (2 Δs + γ Δh),  β = ω/2.
+// Moment form: algebraically the same collision as the oracle's
+// kbc_collide, organised to cut the instruction count:
+//  * the second moments of f^neq come from the populations directly:
+//    sum_i g_i e_ia e_ib = S_ab and sum_i g^eq_i e_ia e_ib = δρ/3 δ_ab +
+//    j_a j_b/ρ (Eq.5 on a lattice with 4th-order isotropy, both D3Q19 and
+//    D3Q27), so N_xz = (S_xx - S_zz) - (j_x² - j_z²)/ρ, N_yz likewise and
+//    Π_ab = S_ab - j_a j_b/ρ for a != b (the δρ/3 terms cancel);
+//  * g^eq is built twice (the entropic products, the update), never stored:
+//    opaque copies of the moments (fresh()) keep the compiler from holding
+//    27 g^eq values live between the passes (occupancy);
+//  * f* = f - β(2Δs + γΔh) with Δh = f^neq - Δs is applied as
+//    g* = g + A (g^eq - g) - B Δs, A = βγ, B = β(2 - γ).
 template <typename T>
 __device__ __forceinline__ void collide_kbc(T (&g)[27], T omega) {
   constexpr int Q = 27;
   T drho = g[0], jx = T(0), jy = T(0), jz = T(0);
+  T sxx = T(0), syy = T(0), szz = T(0), sxy = T(0), sxz = T(0), syz = T(0);
 #pragma unroll
   for (int q = 1; q < Q; q += 2) {
-    const T sm = g[q] + g[q + 1];
+    const T sm = g[q] + g[q + 1];  // e_a e_b is even in e: pair sums
     const T df = g[q] - g[q + 1];
     drho += sm;
     if (ex(q) > 0) jx += df; else if (ex(q) < 0) jx -= df;
     if (ey(q) > 0) jy += df; else if (ey(q) < 0) jy -= df;
     if (ez(q) > 0) jz += df; else if (ez(q) < 0) jz -= df;
+    if (ex(q)) sxx += sm;
+    if (ey(q)) syy += sm;
+    if (ez(q)) szz += sm;
+    if (ex(q) * ey(q) > 0) sxy += sm; else if (ex(q) * ey(q) < 0) sxy -= sm;
+    if (ex(q) * ez(q) > 0) sxz += sm; else if (ex(q) * ez(q) < 0) sxz -= sm;
+    if (ey(q) * ez(q) > 0) syz += sm; else if (ey(q) * ez(q) < 0) syz -= sm;
   }
   const T inv = recip<T>(T(1) + drho);
-  const T base0 = drho - T(1.5) * (jx * jx + jy * jy + jz * jz) * inv;  // g^eq = w (base + 3 e.j + 4.5 (e.j)^2 / rho)
+  const T jxi = jx * inv, jyi = jy * inv, jzi = jz * inv;
+  const T nxz = (sxx - szz) - (jx * jxi - jz * jzi);
+  const T nyz = (syy - szz) - (jy * jyi - jz * jzi);
+  const T sixth = T(1) / T(6);
+  const T sx = (T(2) * nxz - nyz) * sixth, sy = (T(2) * nyz - nxz) * sixth, sz = -(nxz + nyz) * sixth;
+  const T exy = (sxy - jx * jyi) * T(0.25), exz = (sxz - jx * jzi) * T(0.25), eyz = (syz - jy * jzi) * T(0.25);
+  const T base0 = drho - T(1.5) * (jx * jxi + jy * jyi + jz * jzi);  // g^eq = w (base + 3 e.j + 4.5 (e.j)^2 / ρ)
   const T c450 = T(4.5) * inv;
-  // g^eq of the pair (q, q+1): sym ± asym
   auto geq_pair = [](int q, T base, T c45, T x, T y, T z, T& sym, T& asym) {
     T ej = T(0);
     if (ex(q) > 0) ej += x; else if (ex(q) < 0) ej -= x;
@@ -175,31 +208,8 @@ __device__ __forceinline__ void collide_kbc(T (&g)[27], T omega) {
     if (ez(q) > 0) ej += z; else if (ez(q) < 0) ej -= z;
     const T w = T(weight<Q>(q));
     sym = w * (base + c45 * ej * ej);
-    asym = w * T(3) * ej;
+    asym = (w * T(3)) * ej;
   };
-  // pass 1: f^neq in place, second moments of f^neq from pair sums
-  T pxx = 0, pyy = 0, pzz = 0, pxy = 0, pxz = 0, pyz = 0;
-  {
-    const T base = fresh(base0), c45 = fresh(c450), x = fresh(jx), y = fresh(jy), z = fresh(jz);
-    g[0] -= T(weight<Q>(0)) * base;
-#pragma unroll
-    for (int q = 1; q < Q; q += 2) {
-      T sym, asym;
-      geq_pair(q, base, c45, x, y, z, sym, asym);
-      g[q] -= sym + asym;
-      g[q + 1] -= sym - asym;
-      const T ps = g[q] + g[q + 1];
-      if (ex(q)) pxx += ps;
-      if (ey(q)) pyy += ps;
-      if (ez(q)) pzz += ps;
-      if (ex(q) * ey(q) > 0) pxy += ps; else if (ex(q) * ey(q) < 0) pxy -= ps;
-      if (ex(q) * ez(q) > 0) pxz += ps; else if (ex(q) * ez(q) < 0) pxz -= ps;
-      if (ey(q) * ez(q) > 0) pyz += ps; else if (ey(q) * ez(q) < 0) pyz -= ps;
-    }
-  }
-  const T nxz = pxx - pzz, nyz = pyy - pzz;
-  const T sx = (T(2) * nxz - nyz) / T(6), sy = (-nxz + T(2) * nyz) / T(6), sz = (-nxz - nyz) / T(6);
-  const T exy = pxy / T(4), exz = pxz / T(4), eyz = pyz / T(4);
   auto ds = [&](int q) -> T {
     const int n2 = ex(q) * ex(q) + ey(q) * ey(q) + ez(q) * ez(q);
     if (n2 == 1) return ex(q) ? sx : (ey(q) ? sy : sz);
@@ -210,26 +220,31 @@ __device__ __forceinline__ void collide_kbc(T (&g)[27], T omega) {
     }
     return T(0);
   };
-  // pass 2: <Δs|Δh>, <Δh|Δh> with weights 1/f^eq (two partial sums each:
-  // shorter dependent-add chains for the fp64 pipe)
+  // <Δs|Δh>, <Δh|Δh> with weights 1/f^eq (two partial sums each)
   T sh = 0, hh = 0, sh2 = 0, hh2 = 0;
   {
     const T base = fresh(base0), c45 = fresh(c450), x = fresh(jx), y = fresh(jy), z = fresh(jz);
     {
-      const T ifeq = recip<T>(T(weight<Q>(0)) * (T(1) + base));
-      const T h = g[0];
-      hh += h * h * ifeq;
+      const T geq0 = T(weight<Q>(0)) * base;
+      const T h = g[0] - geq0;
+      hh += h * h * rcp_feq<T>(T(weight<Q>(0)) + geq0);
     }
 #pragma unroll
     for (int q = 1; q < Q; q += 2) {
       T sym, asym;
       geq_pair(q, base, c45, x, y, z, sym, asym);
-      // one reciprocal per opposite pair: 1/(a+b) = (a-b)/(a²-b²), 1/(a-b) = (a+b)/(a²-b²)
-      const T a = T(weight<Q>(q)) + sym;
-      const T r = recip<T>(a * a - asym * asym);
-      const T i0 = (a - asym) * r, i1 = (a + asym) * r;
+      const T a = T(weight<Q>(q)) + sym;  // f^eq = a ± asym
+      T i0, i1;
+      if constexpr (sizeof(T) == 4) {
+        i0 = rcp_feq<T>(a + asym);
+        i1 = rcp_feq<T>(a - asym);
+      } else {  // one rounded reciprocal per pair: 1/(a±b) = (a∓b)/(a²-b²)
+        const T r = recip<T>(a * a - asym * asym);
+        i0 = (a - asym) * r;
+        i1 = (a + asym) * r;
+      }
       const T s0 = ds(q), s1 = ds(q + 1);
-      const T h0 = g[q] - s0, h1 = g[q + 1] - s1;
+      const T h0 = (g[q] - (sym + asym)) - s0, h1 = (g[q + 1] - (sym - asym)) - s1;
       sh += s0 * h0 * i0;
       hh += h0 * h0 * i0;
       sh2 += s1 * h1 * i1;
@@ -240,18 +255,20 @@ __device__ __forceinline__ void collide_kbc(T (&g)[27], T omega) {
   hh += hh2;
   const T beta = omega / T(2);
   const T gamma = (hh < T(1e-30)) ? T(2) : T(1) / beta - (T(2) - T(1) / beta) * sh / hh;
-  // pass 3: f* = f^eq + f^neq - β (2 Δs + γ Δh)
+  const T A = beta * gamma, B = beta * (T(2) - gamma);
   {
     const T base = fresh(base0), c45 = fresh(c450), x = fresh(jx), y = fresh(jy), z = fresh(jz);
-    g[0] = T(weight<Q>(0)) * base + g[0] - beta * (gamma * g[0]);
+    g[0] += A * (T(weight<Q>(0)) * base - g[0]);
 #pragma unroll
     for (int q = 1; q < Q; q += 2) {
       T sym, asym;
       geq_pair(q, base, c45, x, y, z, sym, asym);
-      const T s0 = ds(q), s1 = ds(q + 1);
-      const T h0 = g[q] - s0, h1 = g[q + 1] - s1;
-      g[q] = (sym + asym) + g[q] - beta * (T(2) * s0 + gamma * h0);
-      g[q + 1] = (sym - asym) + g[q + 1] - beta * (T(2) * s1 + gamma * h1);
+      g[q] += A * ((sym + asym) - g[q]);
+      g[q + 1] += A * ((sym - asym) - g[q + 1]);
+      if (ex(q) * ex(q) + ey(q) * ey(q) + ez(q) * ez(q) < 3) {  // Δs = 0 on corner directions
+        g[q] -= B * ds(q);
+        g[q + 1] -= B * ds(q + 1);
+      }
     }
   }
 }
