@@ -696,7 +696,11 @@ __device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t
   // instruction-cache misses with the long collision); BGK: separate sites,
   // so the plain path keeps its own spill-free register assignment
   constexpr bool kShared = (COLL == LBM_KBC);
+#ifdef LBMR_DEBUG_ALLPLAIN
+  if (true) {  // timing experiment only (wrong results): every warp takes the plain path
+#else
   if (fm == FULL && sm == 0u) {
+#endif
     pull_all<Q, T, false>(g, P.src, G, rec, blk, true, std::make_integer_sequence<int, Q>{});
     if (!kShared) {
       if (COLLIDE) collide<Q, COLL, T>(g, P.omega);

@@ -118,6 +118,64 @@ def test_T2_kbc_gamma2_is_bgk_and_shear_relaxes_at_omega():
         assert np.abs(fs - b).max() > 0
 
 
+@pytest.mark.parametrize("Q", [19, 27])
+def test_T2_equilibrium_second_moment_closed_form(Q):
+    """Eq.(5) on a lattice with 4th-order isotropy: sum_i f^eq_i e_ia e_ib =
+    rho/3 delta_ab + rho u_a u_b exactly (the identity the CUDA KBC uses to
+    take the f^neq second moments straight from the populations)."""
+    e, w, _ = oracle.lattice(Q)
+    rng = np.random.default_rng(11)
+    for _ in range(20):
+        rho = rng.uniform(0.8, 1.2)
+        u = rng.uniform(-0.1, 0.1, 3)
+        feq = oracle.equilibrium(Q, rho, u)
+        P = np.einsum("i,ia,ib->ab", feq, e, e)
+        assert np.abs(P - (rho / 3 * np.eye(3) + rho * np.outer(u, u))).max() < 2e-16
+
+
+def _kbc_moment_form(e, w, f, om):
+    """The CUDA path's KBC arrangement (level_step.cu collide_kbc), restated in
+    numpy on plain populations: second moments of f^neq from f and the closed
+    form above, then f* = f + A (f^eq - f) - B ds with A = beta gamma,
+    B = beta (2 - gamma).  Shares nothing with the oracle but Eq.(5)'s closed
+    form and the lattice table."""
+    rho = f.sum()
+    j = e.T @ f
+    S = np.einsum("i,ia,ib->ab", f, e, e)
+    Pneq = S - (rho / 3 * np.eye(3) + np.outer(j, j) / rho)
+    nxz, nyz = Pneq[0, 0] - Pneq[2, 2], Pneq[1, 1] - Pneq[2, 2]
+    ax = np.array([(2 * nxz - nyz) / 6, (-nxz + 2 * nyz) / 6, (-nxz - nyz) / 6])
+    ds = np.zeros(len(f))
+    for i, c in enumerate(e):
+        n2 = int((c * c).sum())
+        if n2 == 1:
+            ds[i] = ax[int(np.flatnonzero(c)[0])]
+        elif n2 == 2:
+            a, b = np.flatnonzero(c)
+            ds[i] = c[a] * c[b] * Pneq[a, b] / 4
+    u = j / rho
+    eu = e @ u
+    feq = w * rho * (1 + 3 * eu + 4.5 * eu ** 2 - 1.5 * u @ u)
+    h = (f - feq) - ds
+    sh, hh = np.sum(ds * h / feq), np.sum(h * h / feq)
+    beta = om / 2
+    gamma = 2.0 if hh < 1e-30 else 1 / beta - (2 - 1 / beta) * sh / hh
+    return f + beta * gamma * (feq - f) - beta * (2 - gamma) * ds
+
+
+def test_T2_kbc_moment_form_equals_oracle_kbc():
+    """The reformulated KBC the CUDA kernel computes equals the oracle's
+    step-by-step R-A9 collision to rounding (random states, several omega)."""
+    Q = 27
+    e, w, _ = oracle.lattice(Q)
+    rng = np.random.default_rng(12)
+    for _ in range(30):
+        f = _random_f(Q, rng, amp=0.1)
+        om = rng.uniform(1.0, 1.999)
+        ref = oracle.collide_cell(Q, "kbc", om, f)
+        assert np.abs(_kbc_moment_form(e.astype(float), w, f, om) - ref).max() < 1e-15
+
+
 def test_T2_kbc_matches_brute_numpy_kbc():
     from oracle.brute import collide, lattice as blat
     e_o, w_o, _ = oracle.lattice(27)
