@@ -360,14 +360,19 @@ __device__ __forceinline__ void resolve_slow_sv(const StepParams<T>& P, T* sv, u
 }
 
 template <int Q, typename T>
-__device__ __forceinline__ void resolve_slow(const StepParams<T>& P, T (&g)[Q], uint32_t slow, unsigned j, int blk,
-                                             int t) {
+__device__ __forceinline__ void resolve_slow_links(const StepParams<T>& P, uint32_t slow, unsigned j, int blk, int t) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
-  T* sv = reinterpret_cast<T*>(smem_raw) + threadIdx.x;
-  resolve_slow_sv<Q, T>(P, sv, slow, j, blk, t);
+  resolve_slow_sv<Q, T>(P, reinterpret_cast<T*>(smem_raw) + threadIdx.x, slow, j, blk, t);
+}
+
+// g[q] = this thread's column entry q for every q of the mask
+template <int Q, typename T>
+__device__ __forceinline__ void merge_column(T (&g)[Q], uint32_t mask) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  const T* sv = reinterpret_cast<const T*>(smem_raw) + threadIdx.x;
 #pragma unroll
-  for (int q = 0; q < Q; ++q)
-    if (slow & (1u << q)) g[q] = sv[q * 256];
+  for (int q = 1; q < Q; ++q)
+    if ((mask >> q) & 1u) g[q] = sv[q * 256];
 }
 
 // ---------------------------------------------------------------- fused kernel
@@ -475,9 +480,11 @@ __device__ __forceinline__ void pull_all(T (&g)[Q], const T* __restrict__ src, c
 // speculatively from the block arithmetic's source.  bounce_issue() fetches
 // the cell's own post-collision opposite populations (halfway bounce-back,
 // P:L264) with cp.async straight into this thread's column of the shared
-// staging buffer — all in flight together and without holding registers
-// while the main pulls are in flight; apply_bounce() merges them and adds
-// the BC term.
+// staging buffer — for every direction of the warp's bounce-mask union
+// (record word kRecBounce), issued before the cell's own info has arrived,
+// all in flight together with the pulls and without holding registers;
+// merge_column() takes the cell's own bounce links from the column and
+// bounce_fix() adds the BC term.
 template <int Q, typename T>
 __device__ __forceinline__ void bounce_issue(const StepParams<T>& P, uint32_t bounce, unsigned own) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -492,20 +499,6 @@ __device__ __forceinline__ void bounce_issue(const StepParams<T>& P, uint32_t bo
     }
   }
   asm volatile("cp.async.commit_group;" ::: "memory");
-}
-
-template <int Q, typename T>
-__device__ __forceinline__ void bounce_fix(const StepParams<T>& P, T (&g)[Q], uint32_t bounce, unsigned key);
-
-template <int Q, typename T>
-__device__ __forceinline__ void apply_bounce(const StepParams<T>& P, T (&g)[Q], uint32_t bounce, unsigned key) {
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  const T* sv = reinterpret_cast<const T*>(smem_raw) + threadIdx.x;
-  asm volatile("cp.async.wait_all;" ::: "memory");
-#pragma unroll
-  for (int q = 1; q < Q; ++q)
-    if ((bounce >> q) & 1u) g[q] = sv[q * 256];
-  bounce_fix<Q, T>(P, g, bounce, key);
 }
 
 // BC term of the bounce links: NOSLIP keeps the bounced value, VELOCITY adds
@@ -712,15 +705,24 @@ __device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t
     const int slot = __shfl_sync(FULL, rec, kRecSlot);
     const bool fluid = (fm >> lane) & 1u;
     const bool special = (sm >> lane) & 1u;
+    // bounce-back sources (the cell's own opposite populations) of every
+    // direction some cell of this warp bounces: copied into the thread's
+    // shared-memory column right away, so they travel with the pulls instead
+    // of after the cell's info arrives
+    const uint32_t bm = fluid ? (uint32_t)__ldg(R + kRecBounce + (t >> 5)) : 0u;
     uint4 ci = make_uint4(0u, 0u, 0u, kNoBCSource);
     if (special) ci = __ldg(P.cellinfo + (unsigned)slot * kCells + t);
+#ifndef LBMR_DEBUG_NOSLOW
+    if (bm) bounce_issue<Q, T>(P, bm, own);
+#endif
     pull_all<Q, T, true>(g, P.src, G, rec, blk, fluid, std::make_integer_sequence<int, Q>{});
     if (!fluid) return;
 #ifndef LBMR_DEBUG_NOSLOW
-    if (ci.z) bounce_issue<Q, T>(P, ci.z, own);
-    if (ci.z) apply_bounce<Q, T>(P, g, ci.z, ci.w);
+    if (bm) asm volatile("cp.async.wait_all;" ::: "memory");
     const uint32_t recs = ci.x & ((1u << Q) - 1u);
-    if (recs) resolve_slow<Q, T>(P, g, recs, ci.y, blk, t);
+    if (recs) resolve_slow_links<Q, T>(P, recs, ci.y, blk, t);  // into the column, disjoint from ci.z
+    if (ci.z | recs) merge_column<Q, T>(g, ci.z | recs);
+    if (ci.z) bounce_fix<Q, T>(P, g, ci.z, ci.w);
 #endif
   }
   if (COLLIDE) collide<Q, COLL, T>(g, P.omega);
