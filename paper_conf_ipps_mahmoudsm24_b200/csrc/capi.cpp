@@ -54,6 +54,7 @@ struct DevLevel {
   int32_t* nbr = nullptr;
   int32_t* special_slot = nullptr;
   uint32_t* cellinfo = nullptr;
+  uint32_t* bmask = nullptr;
   uint32_t* links = nullptr;
   uint32_t* coal = nullptr;
   int32_t* bpeer = nullptr;
@@ -186,6 +187,7 @@ StepParams<T> make_params(const lbm_grid* g, int L, int64_t k) {
   p.nbr = D.nbr;
   p.special_slot = D.special_slot;
   p.cellinfo = reinterpret_cast<const uint4*>(D.cellinfo);
+  p.bmask = D.bmask;
   p.links = reinterpret_cast<const uint2*>(D.links);
   p.coal = D.coal;
   p.origin = D.origin;
@@ -624,6 +626,7 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     if ((s = dev_upload(g, &D.nbr, H.nbr))) return cleanup(s);
     if ((s = dev_upload(g, &D.special_slot, H.special_slot))) return cleanup(s);
     if ((s = dev_upload(g, &D.cellinfo, H.cellinfo))) return cleanup(s);
+    if ((s = dev_upload(g, &D.bmask, H.bmask))) return cleanup(s);
     if ((s = dev_upload(g, &D.links, H.links))) return cleanup(s);
     if ((s = dev_upload(g, &D.coal, H.coal))) return cleanup(s);
     if ((s = dev_upload(g, &D.bpeer, H.bpeer))) return cleanup(s);
@@ -640,6 +643,7 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     // the dense per-level tables are on the device now; keep only counters
     // (the host block map is kept for lbm_probe)
     std::vector<uint32_t>().swap(H.cellinfo);
+    std::vector<uint32_t>().swap(H.bmask);
     std::vector<uint32_t>().swap(H.links);
     std::vector<uint32_t>().swap(H.coal);
     std::vector<int32_t>().swap(H.nbr);

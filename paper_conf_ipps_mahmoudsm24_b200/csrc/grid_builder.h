@@ -23,6 +23,7 @@ struct HostLevel {
   std::vector<int32_t> nbr;      // [nfluid*kRec] block records (lattice.h: neighbours, slot, origin)
   std::vector<int32_t> special_slot;  // [nfluid] index into cellinfo or -1 (plain block)
   std::vector<uint32_t> cellinfo;     // [nspecial*512][kCellInfoWords] (lattice.h)
+  std::vector<uint32_t> bmask;        // [nspecial][kBounceWords] per-warp union of the bounce masks
   std::vector<uint32_t> links;        // [nlinks][2] slow-link records (lattice.h kLink*)
   std::vector<uint32_t> coal;         // coalescence candidate population indices
   int64_t nlinks = 0;

@@ -30,6 +30,7 @@ struct StepParams {
   const int32_t* nbr;           // [nfluid][kRec] block records (lattice.h)
   const int32_t* special_slot;  // [nfluid]
   const uint4* cellinfo;        // [nspecial][512] lattice.h kCellInfoWords layout
+  const uint32_t* bmask;        // [nspecial][kBounceWords] per-warp bounce-mask unions
   const uint2* links;           // slow-link records (lattice.h kLink*)
   const uint32_t* coal;         // coalescence candidate lists
   const int32_t* origin;        // [nblocks][3] block coordinates

@@ -40,20 +40,20 @@ LBM_HD constexpr int nbr_slot(int dx, int dy, int dz) { return (dx + 1) + 3 * (d
 constexpr int kBlock = 8;            // B = 8 (B compile time)
 constexpr int kCells = 512;          // B^3
 constexpr unsigned kFluidBit = 1u << 31;
-// per-fluid-block record of 80 int32 (one coalesced warp load of the first
-// 128 bytes, broadcast loads of the per-warp words): [0..26] neighbour block
-// ids by nbr_slot (-1: none, outside, or a block without fluid leaves), [27]
-// special slot (-1 plain), [28..30] block coordinates, [31] unused, [32+w]
-// fluid-leaf mask of warp w (cells 32w..32w+31), [48+w] mask of the fluid
-// leaves of warp w that have a slow link, [64+w] union over the fluid leaves
-// of warp w of their bounce masks (cellinfo [2]): the kernel issues the
-// bounce-back copies for these directions before the cell's info arrives
-constexpr int kRec = 80;
+// per-fluid-block record of 64 int32 (two 128-byte lines, one warp load
+// each): [0..26] neighbour block ids by nbr_slot (-1: none, outside, or a
+// block without fluid leaves), [27] special slot (-1 plain), [28..30] block
+// coordinates, [31] unused, [32+w] fluid-leaf mask of warp w (cells 32w..32w+31),
+// [48+w] mask of the fluid leaves of warp w that have a slow link
+constexpr int kRec = 64;
 constexpr int kRecSlot = 27;
 constexpr int kRecOrigin = 28;
 constexpr int kRecFluid = 32;
 constexpr int kRecSpecial = 48;
-constexpr int kRecBounce = 64;
+// per special block: 16 words, word w = union over the fluid leaves of warp w
+// of their bounce masks (cellinfo [2]); the kernel issues the bounce-back
+// copies for these directions before the cell's own info has arrived
+constexpr int kBounceWords = 16;
 
 // per-cell info of a special block (uint4):
 //  [0] bit q = link q resolved through a slow-link record, bit 31 = fluid leaf

@@ -172,15 +172,18 @@ __device__ __forceinline__ T rcp_feq(T x) {
 //    27 g^eq values live between the passes (occupancy);
 //  * f* = f - β(2Δs + γΔh) with Δh = f^neq - Δs is applied as
 //    g* = g + A (g^eq - g) - B Δs, A = βγ, B = β(2 - γ).
-template <typename T>
-__device__ __forceinline__ void collide_kbc(T (&g)[27], T omega) {
+// Populations are read through acc.get(q) and the results written through
+// acc.put(q, v) (KbcRegs: the thread's registers).
+template <typename T, typename Acc>
+__device__ __forceinline__ void collide_kbc_acc(Acc& acc, T omega) {
   constexpr int Q = 27;
-  T drho = g[0], jx = T(0), jy = T(0), jz = T(0);
+  T drho = acc.get(0), jx = T(0), jy = T(0), jz = T(0);
   T sxx = T(0), syy = T(0), szz = T(0), sxy = T(0), sxz = T(0), syz = T(0);
 #pragma unroll
   for (int q = 1; q < Q; q += 2) {
-    const T sm = g[q] + g[q + 1];  // e_a e_b is even in e: pair sums
-    const T df = g[q] - g[q + 1];
+    const T gq = acc.get(q), gq1 = acc.get(q + 1);
+    const T sm = gq + gq1;  // e_a e_b is even in e: pair sums
+    const T df = gq - gq1;
     drho += sm;
     if (ex(q) > 0) jx += df; else if (ex(q) < 0) jx -= df;
     if (ey(q) > 0) jy += df; else if (ey(q) < 0) jy -= df;
@@ -226,7 +229,7 @@ __device__ __forceinline__ void collide_kbc(T (&g)[27], T omega) {
     const T base = fresh(base0), c45 = fresh(c450), x = fresh(jx), y = fresh(jy), z = fresh(jz);
     {
       const T geq0 = T(weight<Q>(0)) * base;
-      const T h = g[0] - geq0;
+      const T h = acc.get(0) - geq0;
       hh += h * h * rcp_feq<T>(T(weight<Q>(0)) + geq0);
     }
 #pragma unroll
@@ -244,7 +247,7 @@ __device__ __forceinline__ void collide_kbc(T (&g)[27], T omega) {
         i1 = (a + asym) * r;
       }
       const T s0 = ds(q), s1 = ds(q + 1);
-      const T h0 = (g[q] - (sym + asym)) - s0, h1 = (g[q + 1] - (sym - asym)) - s1;
+      const T h0 = (acc.get(q) - (sym + asym)) - s0, h1 = (acc.get(q + 1) - (sym - asym)) - s1;
       sh += s0 * h0 * i0;
       hh += h0 * h0 * i0;
       sh2 += s1 * h1 * i1;
@@ -258,19 +261,38 @@ __device__ __forceinline__ void collide_kbc(T (&g)[27], T omega) {
   const T A = beta * gamma, B = beta * (T(2) - gamma);
   {
     const T base = fresh(base0), c45 = fresh(c450), x = fresh(jx), y = fresh(jy), z = fresh(jz);
-    g[0] += A * (T(weight<Q>(0)) * base - g[0]);
+    {
+      const T g0 = acc.get(0);
+      acc.put(0, g0 + A * (T(weight<Q>(0)) * base - g0));
+    }
 #pragma unroll
     for (int q = 1; q < Q; q += 2) {
       T sym, asym;
       geq_pair(q, base, c45, x, y, z, sym, asym);
-      g[q] += A * ((sym + asym) - g[q]);
-      g[q + 1] += A * ((sym - asym) - g[q + 1]);
+      const T gq = acc.get(q), gq1 = acc.get(q + 1);
+      T r0 = gq + A * ((sym + asym) - gq);
+      T r1 = gq1 + A * ((sym - asym) - gq1);
       if (ex(q) * ex(q) + ey(q) * ey(q) + ez(q) * ez(q) < 3) {  // Δs = 0 on corner directions
-        g[q] -= B * ds(q);
-        g[q + 1] -= B * ds(q + 1);
+        r0 -= B * ds(q);
+        r1 -= B * ds(q + 1);
       }
+      acc.put(q, r0);
+      acc.put(q + 1, r1);
     }
   }
+}
+
+template <typename T>
+struct KbcRegs {
+  T (&g)[27];
+  __device__ __forceinline__ T get(int q) const { return g[q]; }
+  __device__ __forceinline__ void put(int q, T v) { g[q] = v; }
+};
+
+template <typename T>
+__device__ __forceinline__ void collide_kbc(T (&g)[27], T omega) {
+  KbcRegs<T> a{g};
+  collide_kbc_acc<T>(a, omega);
 }
 
 template <int Q, int COLL, typename T>
@@ -481,7 +503,7 @@ __device__ __forceinline__ void pull_all(T (&g)[Q], const T* __restrict__ src, c
 // the cell's own post-collision opposite populations (halfway bounce-back,
 // P:L264) with cp.async straight into this thread's column of the shared
 // staging buffer — for every direction of the warp's bounce-mask union
-// (record word kRecBounce), issued before the cell's own info has arrived,
+// (lattice.h kBounceWords), issued before the cell's own info has arrived,
 // all in flight together with the pulls and without holding registers;
 // merge_column() takes the cell's own bounce links from the column and
 // bounce_fix() adds the BC term.
@@ -674,6 +696,12 @@ __device__ __forceinline__ void halo_store(const StepParams<T>& P, const T (&g)[
 // (host-checked: nblocks * Q * 512 < 2^32).
 // COLLIDE = false: the stream-only half S_L^k of the unfused schedule
 // (lbm_set_schedule): the pulled post-streaming populations are stored as is.
+// Bounce copies issued with the pulls (per-warp union masks, lattice.h
+// kBounceWords) or after the cell's info: measured per lattice — D3Q27
+// (cfg4: every warp walls) +3 % BGK, +20 % KBC; D3Q19 (cfg5) -0.4 %.
+template <int Q>
+constexpr bool kEarlyBounce = (Q == 27);
+
 template <int Q, int COLL, typename T, bool HALO, bool COLLIDE = true>
 __device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t) {
   constexpr unsigned FULL = 0xffffffffu;
@@ -705,25 +733,47 @@ __device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t
     const int slot = __shfl_sync(FULL, rec, kRecSlot);
     const bool fluid = (fm >> lane) & 1u;
     const bool special = (sm >> lane) & 1u;
-    // bounce-back sources (the cell's own opposite populations) of every
-    // direction some cell of this warp bounces: copied into the thread's
-    // shared-memory column right away, so they travel with the pulls instead
-    // of after the cell's info arrives
-    const uint32_t bm = fluid ? (uint32_t)__ldg(R + kRecBounce + (t >> 5)) : 0u;
-    uint4 ci = make_uint4(0u, 0u, 0u, kNoBCSource);
-    if (special) ci = __ldg(P.cellinfo + (unsigned)slot * kCells + t);
+    if constexpr (kEarlyBounce<Q>) {
+      // bounce-back sources (the cell's own opposite populations) of every
+      // direction some cell of this warp bounces: copied into the thread's
+      // shared-memory column right after the pulls, not after the cell's
+      // info arrives (partly fluid warps without special cells skip the
+      // load: sm is warp-uniform)
+      const uint32_t bm = (sm != 0u && fluid) ? __ldg(P.bmask + (unsigned)slot * kBounceWords + (t >> 5)) : 0u;
+      pull_all<Q, T, true>(g, P.src, G, rec, blk, fluid, std::make_integer_sequence<int, Q>{});
 #ifndef LBMR_DEBUG_NOSLOW
-    if (bm) bounce_issue<Q, T>(P, bm, own);
+      if (bm) bounce_issue<Q, T>(P, bm, own);
 #endif
-    pull_all<Q, T, true>(g, P.src, G, rec, blk, fluid, std::make_integer_sequence<int, Q>{});
-    if (!fluid) return;
+      if (!fluid) return;
+      uint4 ci = make_uint4(0u, 0u, 0u, kNoBCSource);
+      if (special) ci = __ldg(P.cellinfo + (unsigned)slot * kCells + t);
 #ifndef LBMR_DEBUG_NOSLOW
-    if (bm) asm volatile("cp.async.wait_all;" ::: "memory");
-    const uint32_t recs = ci.x & ((1u << Q) - 1u);
-    if (recs) resolve_slow_links<Q, T>(P, recs, ci.y, blk, t);  // into the column, disjoint from ci.z
-    if (ci.z | recs) merge_column<Q, T>(g, ci.z | recs);
-    if (ci.z) bounce_fix<Q, T>(P, g, ci.z, ci.w);
+      if (bm) asm volatile("cp.async.wait_all;" ::: "memory");
+      const uint32_t recs = ci.x & ((1u << Q) - 1u);
+      if (recs) resolve_slow_links<Q, T>(P, recs, ci.y, blk, t);  // into the column, disjoint from ci.z
+      if (ci.z | recs) merge_column<Q, T>(g, ci.z | recs);
+      if (ci.z) bounce_fix<Q, T>(P, g, ci.z, ci.w);
 #endif
+    } else {
+      // the cell's info first, its bounce copies once it has arrived
+      uint4 ci = make_uint4(0u, 0u, 0u, kNoBCSource);
+      if (special) ci = __ldg(P.cellinfo + (unsigned)slot * kCells + t);
+      pull_all<Q, T, true>(g, P.src, G, rec, blk, fluid, std::make_integer_sequence<int, Q>{});
+      if (!fluid) return;
+#ifndef LBMR_DEBUG_NOSLOW
+      if (ci.z) {
+        bounce_issue<Q, T>(P, ci.z, own);
+        asm volatile("cp.async.wait_all;" ::: "memory");
+        merge_column<Q, T>(g, ci.z);
+        bounce_fix<Q, T>(P, g, ci.z, ci.w);
+      }
+      const uint32_t recs = ci.x & ((1u << Q) - 1u);
+      if (recs) {
+        resolve_slow_links<Q, T>(P, recs, ci.y, blk, t);
+        merge_column<Q, T>(g, recs);
+      }
+#endif
+    }
   }
   if (COLLIDE) collide<Q, COLL, T>(g, P.omega);
   store_cell<Q, T>(g, P.dst, blk, t);
