@@ -150,7 +150,7 @@ def run_reference(args, ws, rank):
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": "MLUPS", "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3 / args.steps,
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
         "data": "synthetic", "config": {"workload": CONFIGS[args.config][1], "sample": sample},
         "cpu_baseline": {"value": value, "unit": "MLUPS", "cores": cores, "kind": "oracle",
                          "sample": f"{sample}; one oracle coarse step per timed step"},
