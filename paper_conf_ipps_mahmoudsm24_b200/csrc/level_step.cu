@@ -318,7 +318,7 @@ __device__ __forceinline__ int opp_rt(int q) { return q == 0 ? 0 : ((q & 1) ? q 
 
 // Values go to this thread's column sv[q * 256] of a shared buffer
 // (conflict-free for any q per lane).
-template <int Q, typename T>
+template <int Q, typename T, int NT = 256>
 __device__ __forceinline__ void resolve_slow_sv(const StepParams<T>& P, T* sv, uint32_t slow, unsigned j, int blk,
                                                 int t) {
   const unsigned own = (unsigned)blk * (unsigned)(Q * kCells) + (unsigned)t;
@@ -376,25 +376,25 @@ __device__ __forceinline__ void resolve_slow_sv(const StepParams<T>& P, T* sv, u
         for (unsigned m = 0; m < n; ++m) acc += __ldg(P.fb + __ldg(c + m));
         val = acc / T(2 * n);
       }
-      sv[q * 256] = val;
+      sv[q * NT] = val;
     }
   }
 }
 
-template <int Q, typename T>
+template <int Q, typename T, int NT = 256>
 __device__ __forceinline__ void resolve_slow_links(const StepParams<T>& P, uint32_t slow, unsigned j, int blk, int t) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
-  resolve_slow_sv<Q, T>(P, reinterpret_cast<T*>(smem_raw) + threadIdx.x, slow, j, blk, t);
+  resolve_slow_sv<Q, T, NT>(P, reinterpret_cast<T*>(smem_raw) + threadIdx.x, slow, j, blk, t);
 }
 
 // g[q] = this thread's column entry q for every q of the mask
-template <int Q, typename T>
+template <int Q, typename T, int NT = 256>
 __device__ __forceinline__ void merge_column(T (&g)[Q], uint32_t mask) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const T* sv = reinterpret_cast<const T*>(smem_raw) + threadIdx.x;
 #pragma unroll
   for (int q = 1; q < Q; ++q)
-    if ((mask >> q) & 1u) g[q] = sv[q * 256];
+    if ((mask >> q) & 1u) g[q] = sv[q * NT];
 }
 
 // ---------------------------------------------------------------- fused kernel
@@ -507,7 +507,7 @@ __device__ __forceinline__ void pull_all(T (&g)[Q], const T* __restrict__ src, c
 // all in flight together with the pulls and without holding registers;
 // merge_column() takes the cell's own bounce links from the column and
 // bounce_fix() adds the BC term.
-template <int Q, typename T>
+template <int Q, typename T, int NT = 256>
 __device__ __forceinline__ void bounce_issue(const StepParams<T>& P, uint32_t bounce, unsigned own) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const unsigned sv = (unsigned)__cvta_generic_to_shared(reinterpret_cast<T*>(smem_raw) + threadIdx.x);
@@ -515,7 +515,7 @@ __device__ __forceinline__ void bounce_issue(const StepParams<T>& P, uint32_t bo
   for (int q = 1; q < Q; ++q) {
     if ((bounce >> q) & 1u) {
       const T* a = P.src + opp(q) * kCells + own;
-      asm volatile("cp.async.ca.shared.global [%0], [%1], %2;" ::"r"(sv + (unsigned)(q * 256 * sizeof(T))), "l"(a),
+      asm volatile("cp.async.ca.shared.global [%0], [%1], %2;" ::"r"(sv + (unsigned)(q * NT * sizeof(T))), "l"(a),
                    "n"(sizeof(T))
                    : "memory");
     }
@@ -702,7 +702,7 @@ __device__ __forceinline__ void halo_store(const StepParams<T>& P, const T (&g)[
 template <int Q>
 constexpr bool kEarlyBounce = (Q == 27);
 
-template <int Q, int COLL, typename T, bool HALO, bool COLLIDE = true>
+template <int Q, int COLL, typename T, bool HALO, bool COLLIDE = true, int NT = 256>
 __device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t) {
   constexpr unsigned FULL = 0xffffffffu;
   const int lane = threadIdx.x & 31;
@@ -742,7 +742,7 @@ __device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t
       const uint32_t bm = (sm != 0u && fluid) ? __ldg(P.bmask + (unsigned)slot * kBounceWords + (t >> 5)) : 0u;
       pull_all<Q, T, true>(g, P.src, G, rec, blk, fluid, std::make_integer_sequence<int, Q>{});
 #ifndef LBMR_DEBUG_NOSLOW
-      if (bm) bounce_issue<Q, T>(P, bm, own);
+      if (bm) bounce_issue<Q, T, NT>(P, bm, own);
 #endif
       if (!fluid) return;
       uint4 ci = make_uint4(0u, 0u, 0u, kNoBCSource);
@@ -750,8 +750,8 @@ __device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t
 #ifndef LBMR_DEBUG_NOSLOW
       if (bm) asm volatile("cp.async.wait_all;" ::: "memory");
       const uint32_t recs = ci.x & ((1u << Q) - 1u);
-      if (recs) resolve_slow_links<Q, T>(P, recs, ci.y, blk, t);  // into the column, disjoint from ci.z
-      if (ci.z | recs) merge_column<Q, T>(g, ci.z | recs);
+      if (recs) resolve_slow_links<Q, T, NT>(P, recs, ci.y, blk, t);  // into the column, disjoint from ci.z
+      if (ci.z | recs) merge_column<Q, T, NT>(g, ci.z | recs);
       if (ci.z) bounce_fix<Q, T>(P, g, ci.z, ci.w);
 #endif
     } else {
@@ -762,15 +762,15 @@ __device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t
       if (!fluid) return;
 #ifndef LBMR_DEBUG_NOSLOW
       if (ci.z) {
-        bounce_issue<Q, T>(P, ci.z, own);
+        bounce_issue<Q, T, NT>(P, ci.z, own);
         asm volatile("cp.async.wait_all;" ::: "memory");
-        merge_column<Q, T>(g, ci.z);
+        merge_column<Q, T, NT>(g, ci.z);
         bounce_fix<Q, T>(P, g, ci.z, ci.w);
       }
       const uint32_t recs = ci.x & ((1u << Q) - 1u);
       if (recs) {
-        resolve_slow_links<Q, T>(P, recs, ci.y, blk, t);
-        merge_column<Q, T>(g, recs);
+        resolve_slow_links<Q, T, NT>(P, recs, ci.y, blk, t);
+        merge_column<Q, T, NT>(g, recs);
       }
 #endif
     }
@@ -798,36 +798,36 @@ __device__ __forceinline__ void collide_cell(const StepParams<T>& P, int blk, in
   if (HALO) halo_store<Q, T>(P, g, blk, t);
 }
 
-// LBMR_CTA512: one CTA per 8^3 block (512 threads) instead of per half block
-#ifndef LBMR_CTA512
-#define LBMR_CTA512 0
+// CTA size of the fused single-rank kernel per variant: a quarter of an 8^3
+// block (128 threads) instead of a half (256); the CTAs per SM scale so the
+// register budget (PlainOcc, in 256-thread units) is unchanged.  The finer
+// CTA granularity measured +1.5-2 % on cfg5 / cfg3 / uniform512 (D3Q19), +5-6 %
+// on the D3Q27 KBC / BGK workloads (fewer warps idle behind a CTA's slowest
+// warp at the end of its life, more CTAs in flight per SM).
+#ifndef LBMR_NT_KBCD
+#define LBMR_NT_KBCD 128
 #endif
-constexpr int kStepThreads = LBMR_CTA512 ? 512 : 256;
-
-#ifndef LBMR_FILL_FIRST
-#define LBMR_FILL_FIRST 0
+#ifndef LBMR_NT_OTHER
+#define LBMR_NT_OTHER 128
 #endif
 template <int Q, int COLL, typename T>
-__global__ void __launch_bounds__(kStepThreads, (PlainOcc<Q, T, COLL>::value * 256) / kStepThreads)
+struct StepCta {
+  static constexpr int threads = (COLL == LBM_KBC && sizeof(T) == 8) ? LBMR_NT_KBCD : LBMR_NT_OTHER;
+  static constexpr int per_block = kCells / threads;
+  static constexpr int min_blocks = (PlainOcc<Q, T, COLL>::value * 256) / threads;
+};
+
+template <int Q, int COLL, typename T>
+__global__ void __launch_bounds__(StepCta<Q, COLL, T>::threads, StepCta<Q, COLL, T>::min_blocks)
     level_step_all(const StepParams<T> P) {
-#if LBMR_FILL_FIRST
-  // leading CTAs refresh the explosion ghosts (they overlap the first wave)
-  const int lead = (trail_items(P.nghost, P.nvfill) + kStepThreads - 1) / kStepThreads;
-  if ((int)blockIdx.x < lead) {
-    trail_fill<Q, T>(P, (int)blockIdx.x * kStepThreads + threadIdx.x);
-    return;
-  }
-  const int b = (int)blockIdx.x - lead;
-#else
-  const int main = P.nfluid * 512 / kStepThreads;
+  constexpr int NT = StepCta<Q, COLL, T>::threads, PB = StepCta<Q, COLL, T>::per_block;
+  const int main = P.nfluid * PB;
   if ((int)blockIdx.x >= main) {  // trailing CTAs refresh the explosion ghosts
-    trail_fill<Q, T>(P, ((int)blockIdx.x - main) * kStepThreads + threadIdx.x);
+    trail_fill<Q, T>(P, ((int)blockIdx.x - main) * NT + threadIdx.x);
     return;
   }
   const int b = (int)blockIdx.x;
-#endif
-  if (kStepThreads == 512) step_cell<Q, COLL, T, false>(P, b, threadIdx.x);
-  else step_cell<Q, COLL, T, false>(P, b >> 1, ((b & 1) << 8) | threadIdx.x);
+  step_cell<Q, COLL, T, false, true, NT>(P, b / PB, (b % PB) * NT + threadIdx.x);
 }
 
 // Partitioned variant: grid = 2 * max(nfluid, 1) CTAs; the first nbctas run
@@ -1117,8 +1117,10 @@ static void launch_typed(int kind, const void* params, cudaStream_t s) {
   } else if (kind == 4) {
     if (p.nfluid > 0) level_collide_inplace<Q, COLL, T><<<dim3(2 * p.nfluid), block, 0, s>>>(p);
   } else {
-    const int gct = (trail_items(p.nghost, p.nvfill) + kStepThreads - 1) / kStepThreads;
-    level_step_all<Q, COLL, T><<<dim3(p.nfluid * 512 / kStepThreads + gct), dim3(kStepThreads), sm, s>>>(p);
+    constexpr int NT = StepCta<Q, COLL, T>::threads;
+    const int gct = (trail_items(p.nghost, p.nvfill) + NT - 1) / NT;
+    level_step_all<Q, COLL, T><<<dim3(p.nfluid * StepCta<Q, COLL, T>::per_block + gct), dim3(NT),
+                                 (size_t)Q * NT * sizeof(T), s>>>(p);
   }
 }
 
