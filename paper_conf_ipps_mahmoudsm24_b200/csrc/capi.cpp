@@ -215,7 +215,7 @@ StepParams<T> make_params(const lbm_grid* g, int L, int64_t k) {
   if (L > 0) p.gsrc = static_cast<const T*>(g->dev[L - 1].pop[((k + 2) / 2) & 1]);  // C_{L-1}^{ceil((k+1)/2)}
   if (g->n_ranks > 1) {
     const HostLevel& H = g->host[L];
-    p.nbctas = std::max(2 * H.nboundary, 1);
+    p.nbctas = std::max(kHaloCtasPerBlock * H.nboundary, 1);
     p.nboundary = H.nboundary;
     p.flags = g->flags;
     p.bpeer = D.bpeer;

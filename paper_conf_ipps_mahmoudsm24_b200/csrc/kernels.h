@@ -21,6 +21,11 @@ struct BCEntry {
   double u[3];              // wall / inlet velocity
 };
 
+// CTA size of the partitioned (halo-protocol) level kernels: a quarter of an
+// 8^3 block; the host counts the protocol CTAs (nbctas) in these units.
+constexpr int kHaloCtaThreads = 128;
+constexpr int kHaloCtasPerBlock = 512 / kHaloCtaThreads;
+
 // Parameters of one fused level-substep launch F_L^k: stream substep k of
 // level L (pull, with BC, Explosion from L-1 and Coalescence from L+1), then
 // collide substep k+1.

@@ -570,6 +570,7 @@ __device__ __forceinline__ void ghost_fill_one(const StepParams<T>& P, int i) {
 }
 
 __host__ __device__ constexpr int ghost_ctas(int n) { return (n + 255) / 256; }
+__host__ __device__ constexpr int halo_fill_ctas(int n) { return (n + kHaloCtaThreads - 1) / kHaloCtaThreads; }
 
 // Volumetric variant: one gather expression = a population of
 // buffer A, B or C (tag) followed by up to three wall reflections, innermost
@@ -830,7 +831,7 @@ __global__ void __launch_bounds__(StepCta<Q, COLL, T>::threads, StepCta<Q, COLL,
   step_cell<Q, COLL, T, false, true, NT>(P, b / PB, (b % PB) * NT + threadIdx.x);
 }
 
-// Partitioned variant: grid = 2 * max(nfluid, 1) CTAs; the first nbctas run
+// Partitioned variant: grid = 4 * max(nfluid, 1) quarter-block CTAs; the first nbctas run
 // the halo protocol around their work.
 // One thread waits until every neighbour has completed the cut-plane part of
 // all kernels this rank has completed (its bumps of our flag reach our
@@ -845,22 +846,24 @@ __global__ void halo_wait_kernel(const unsigned long long* flags, int nb0, int n
 }
 
 template <int Q, int COLL, typename T, bool STREAM>
-__global__ void __launch_bounds__(256, PlainOcc<Q, T, COLL>::value) level_step_halo(const StepParams<T> P) {
-  const int blk = blockIdx.x >> 1;
-  const int t = ((blockIdx.x & 1) << 8) | threadIdx.x;
-  const int main = 2 * max(P.nfluid, 1);
+__global__ void __launch_bounds__(kHaloCtaThreads, (PlainOcc<Q, T, COLL>::value * 256) / kHaloCtaThreads)
+    level_step_halo(const StepParams<T> P) {
+  constexpr int NT = kHaloCtaThreads, PB = kHaloCtasPerBlock;
+  const int blk = (int)blockIdx.x / PB;
+  const int t = ((int)blockIdx.x % PB) * NT + threadIdx.x;
+  const int main = PB * max(P.nfluid, 1);
   // the wait happened in halo_wait_kernel just before this launch; cut-plane
   // CTAs (which write the neighbour's halo) and ghost-refresh CTAs (which may
   // read L-1 halo cells) count towards this kernel's completion signal
   const bool fill = (int)blockIdx.x >= main;
   const bool proto = (int)blockIdx.x < P.nbctas || fill;
   if (fill) {
-    trail_fill<Q, T>(P, ((int)blockIdx.x - main) * 256 + threadIdx.x);
+    trail_fill<Q, T>(P, ((int)blockIdx.x - main) * NT + threadIdx.x);
   } else if (blk < P.nfluid) {
-    if (STREAM) step_cell<Q, COLL, T, true>(P, blk, t);
+    if (STREAM) step_cell<Q, COLL, T, true, true, NT>(P, blk, t);
     else collide_cell<Q, COLL, T, true>(P, blk, t);
   }
-  if (proto) halo_signal<T>(P, P.nbctas + ghost_ctas(trail_items(P.nghost, P.nvfill)));
+  if (proto) halo_signal<T>(P, P.nbctas + halo_fill_ctas(trail_items(P.nghost, P.nvfill)));
 }
 
 template <int Q, int COLL, typename T>
@@ -1104,9 +1107,10 @@ static void launch_typed(int kind, const void* params, cudaStream_t s) {
   const int gc = ghost_ctas(trail_items(p.nghost, p.nvfill));
   if (p.nbctas > 0) {  // partitioned: always launched (the protocol must run)
     halo_wait_kernel<<<1, 1, 0, s>>>(p.flags, p.has_nb[0], p.has_nb[1]);
-    dim3 grid(2 * std::max(p.nfluid, 1) + gc);
-    if (kind == 1) level_step_halo<Q, COLL, T, false><<<grid, block, 0, s>>>(p);
-    else level_step_halo<Q, COLL, T, true><<<grid, block, sm, s>>>(p);
+    dim3 grid(kHaloCtasPerBlock * std::max(p.nfluid, 1) + halo_fill_ctas(trail_items(p.nghost, p.nvfill)));
+    const size_t hs = (size_t)Q * kHaloCtaThreads * sizeof(T);
+    if (kind == 1) level_step_halo<Q, COLL, T, false><<<grid, dim3(kHaloCtaThreads), 0, s>>>(p);
+    else level_step_halo<Q, COLL, T, true><<<grid, dim3(kHaloCtaThreads), hs, s>>>(p);
     return;
   }
   if (p.nfluid <= 0 && p.nghost <= 0 && p.nvfill <= 0) return;
