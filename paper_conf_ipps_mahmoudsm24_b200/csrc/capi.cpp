@@ -638,7 +638,10 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     if ((s = dev_alloc(g, &D.vtemp, (H.vavg.size() / 36) * g->tsize))) return cleanup(s);
     for (int b = 0; b < 2; ++b) {
       if ((s = dev_alloc(g, &D.pop[b], pop_bytes(g, L)))) return cleanup(s);
-      if (cudaMemset(D.pop[b], 0, pop_bytes(g, L)) != cudaSuccess) return cleanup(fail(LBM_E_CUDA, "memset"));
+      // on the grid's stream: a legacy-stream memset is unordered with a
+      // non-blocking user stream and could land after the first halo stores
+      if (cudaMemsetAsync(D.pop[b], 0, pop_bytes(g, L), g->stream) != cudaSuccess)
+        return cleanup(fail(LBM_E_CUDA, "memset"));
     }
     // the dense per-level tables are on the device now; keep only counters
     // (the host block map is kept for lbm_probe)
@@ -652,7 +655,8 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
   void* p;
   if (g->n_ranks > 1) {  // halo-protocol flags, own allocation so it can be shared by CUDA IPC
     if ((s = dev_alloc(g, &p, 4 * sizeof(unsigned long long)))) return cleanup(s);
-    if (cudaMemset(p, 0, 4 * sizeof(unsigned long long)) != cudaSuccess) return cleanup(fail(LBM_E_CUDA, "memset"));
+    if (cudaMemsetAsync(p, 0, 4 * sizeof(unsigned long long), g->stream) != cudaSuccess)
+      return cleanup(fail(LBM_E_CUDA, "memset"));
     g->flags = static_cast<unsigned long long*>(p);
   }
   if ((s = dev_alloc(g, &p, sizeof(BCEntry) * 256))) return cleanup(s);
@@ -663,6 +667,7 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
   if (cudaMemcpy(g->bc_dev, g->bc_host, sizeof(g->bc_host), cudaMemcpyHostToDevice) != cudaSuccess ||
       cudaMemcpy(g->face_dev, g->face_host, 27, cudaMemcpyHostToDevice) != cudaSuccess)
     return cleanup(fail(LBM_E_CUDA, "upload BC table"));
+  if (cudaStreamSynchronize(g->stream) != cudaSuccess) return cleanup(fail(LBM_E_CUDA, "zero-fill"));
   // populations start as g = 0, i.e. f = w (rest equilibrium, rho = 1)
   g->needs_prologue = true;
   *out = g;
@@ -1209,6 +1214,10 @@ lbm_status lbm_halo_connect(lbm_grid* g, int32_t side, const void* blob, int64_t
   void* f = nullptr;
   if ((s = open_ipc(g, h.flags, &f))) return s;
   g->peer_flags[side] = static_cast<unsigned long long*>(f);
+  // every local write to the buffers the peer stores into (zero-fill, init)
+  // is complete before the caller's barrier lets the peer start stepping
+  CUDA_TRY(cudaStreamSynchronize(g->stream));
+  CUDA_TRY(cudaDeviceSynchronize());
   g->connected[side] = true;
   return LBM_OK;
 }
@@ -1230,6 +1239,8 @@ lbm_status lbm_halo_connect_local(lbm_grid* g, int32_t side, lbm_grid* peer) {
     if ((s = dev_upload(g, &D.peer_cells[side], peer->host[L].halo[1 - side]))) return s;
   }
   g->peer_flags[side] = peer->flags;
+  CUDA_TRY(cudaStreamSynchronize(g->stream));
+  CUDA_TRY(cudaStreamSynchronize(peer->stream));
   g->connected[side] = true;
   return LBM_OK;
 }
