@@ -123,7 +123,13 @@ lbm_status dev_upload(lbm_grid* g, T** dst, const std::vector<T>& src) {
   if (cudaMalloc(&p, bytes) != cudaSuccess) return fail(LBM_E_OOM, "cudaMalloc failed (tables)");
   g->allocs.push_back(p);
   g->device_bytes += (int64_t)bytes;
-  if (!src.empty()) CUDA_TRY(cudaMemcpy(p, src.data(), src.size() * sizeof(T), cudaMemcpyHostToDevice));
+  // on the grid's stream and synchronised: a legacy-stream cudaMemcpy from
+  // pageable memory may return before its DMA lands and is unordered with a
+  // non-blocking user stream
+  if (!src.empty()) {
+    CUDA_TRY(cudaMemcpyAsync(p, src.data(), src.size() * sizeof(T), cudaMemcpyHostToDevice, g->stream));
+    CUDA_TRY(cudaStreamSynchronize(g->stream));
+  }
   *dst = static_cast<T*>(p);
   return LBM_OK;
 }
@@ -664,8 +670,12 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
   if ((s = dev_alloc(g, &p, 32))) return cleanup(s);
   g->face_dev = static_cast<uint8_t*>(p);
   compute_face_classes(g);
-  if (cudaMemcpy(g->bc_dev, g->bc_host, sizeof(g->bc_host), cudaMemcpyHostToDevice) != cudaSuccess ||
-      cudaMemcpy(g->face_dev, g->face_host, 27, cudaMemcpyHostToDevice) != cudaSuccess)
+  // same stream as lbm_set_bc's updates: a legacy-stream copy here could land
+  // after them (pageable cudaMemcpy returns before its DMA completes) and
+  // restore the default edge/corner classes (seen as a missing moving-wall
+  // term on lid edges in rare two-process runs)
+  if (cudaMemcpyAsync(g->bc_dev, g->bc_host, sizeof(g->bc_host), cudaMemcpyHostToDevice, g->stream) != cudaSuccess ||
+      cudaMemcpyAsync(g->face_dev, g->face_host, 27, cudaMemcpyHostToDevice, g->stream) != cudaSuccess)
     return cleanup(fail(LBM_E_CUDA, "upload BC table"));
   if (cudaStreamSynchronize(g->stream) != cudaSuccess) return cleanup(fail(LBM_E_CUDA, "zero-fill"));
   // populations start as g = 0, i.e. f = w (rest equilibrium, rho = 1)
