@@ -1031,7 +1031,9 @@ lbm_status lbm_probe(lbm_grid* g, int32_t L, int64_t n, const int64_t* xyz, doub
   void *dv = nullptr, *hv = nullptr;
   lbm_status s;
   if ((s = scratch_dev(g, bytes, &dv)) || (s = scratch_host(g, bytes, &hv))) return s;
-  CUDA_TRY(cudaStreamSynchronize(g->stream));
+  // no wait for the queued steps here: every scratch user synchronises
+  // before returning, so the pinned buffer is free and the upload, probe and
+  // readback queue behind the step
   std::memcpy(hv, cell.data(), n * sizeof(int64_t));
   int64_t* dc = static_cast<int64_t*>(dv);
   double* dr = reinterpret_cast<double*>(dc + n);
