@@ -107,7 +107,10 @@ lbm_status lbm_grid_create(const lbm_grid_desc* desc, int32_t levels, const uint
 
 /* Define boundary class `bc_class` (2..254): kind and wall velocity u_wall[3]
  * (lattice units of the level the link lives on; NULL = 0).  Takes effect at
- * the next lbm_step.  Undefined classes used by masks/face_bc act as NOSLIP. */
+ * the next lbm_step.  Undefined classes used by masks/face_bc act as NOSLIP.
+ * Asynchronous: the entry and the recomputed edge/corner face classes are
+ * enqueued on the grid's stream as kernel arguments (no host wait, no host
+ * buffer kept), so they apply to steps launched after this call only. */
 lbm_status lbm_set_bc(lbm_grid* g, int32_t bc_class, int32_t kind, const double* u_wall);
 
 /* f = f^eq(rho, u) (Eq.5) on the fluid leaves of `level`.  rho: dense

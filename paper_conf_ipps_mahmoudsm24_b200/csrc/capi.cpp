@@ -693,8 +693,10 @@ lbm_status lbm_set_bc(lbm_grid* g, int32_t cls, int32_t kind, const double* u) {
   g->bc_host[cls].kind = kind;
   for (int a = 0; a < 3; ++a) g->bc_host[cls].u[a] = u ? u[a] : 0.0;
   compute_face_classes(g);
-  CUDA_TRY(cudaMemcpyAsync(g->bc_dev + cls, g->bc_host + cls, sizeof(BCEntry), cudaMemcpyHostToDevice, g->stream));
-  CUDA_TRY(cudaMemcpyAsync(g->face_dev, g->face_host, 27, cudaMemcpyHostToDevice, g->stream));
+  FaceTable ft{};
+  std::memcpy(ft.cls, g->face_host, 27);
+  launch_bc_update(g->bc_dev, cls, g->bc_host[cls], g->face_dev, ft, g->stream);
+  CUDA_TRY(cudaGetLastError());
   return LBM_OK;
 }
 

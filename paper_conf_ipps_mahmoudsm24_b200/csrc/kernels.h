@@ -94,6 +94,14 @@ void launch_vavg(int Q, int precision, const uint32_t* ent, int32_t n, void* A, 
 // cut-plane part of every kernel this rank has completed.
 void launch_halo_wait(const unsigned long long* flags, int nb0, int nb1, cudaStream_t s);
 
+// lbm_set_bc's device update: the BC entry of one class and the 27 face
+// classes travel as kernel arguments (copied at launch), so the host call
+// neither waits for the stream nor keeps a host buffer alive.
+struct FaceTable {
+  uint8_t cls[28];
+};
+void launch_bc_update(BCEntry* bc, int cls, BCEntry e, uint8_t* face_cls, FaceTable ft, cudaStream_t s);
+
 // Force-load every kernel (see level_step.cu).
 void preload_kernels();
 

@@ -1075,6 +1075,15 @@ void launch_vavg(int Q, int precision, const uint32_t* ent, int32_t n, void* A, 
   }
 }
 
+__global__ void bc_update_kernel(BCEntry* bc, int cls, BCEntry e, uint8_t* face_cls, FaceTable ft) {
+  if (threadIdx.x == 0) bc[cls] = e;
+  if (threadIdx.x < 27) face_cls[threadIdx.x] = ft.cls[threadIdx.x];
+}
+
+void launch_bc_update(BCEntry* bc, int cls, BCEntry e, uint8_t* face_cls, FaceTable ft, cudaStream_t s) {
+  bc_update_kernel<<<1, 32, 0, s>>>(bc, cls, e, face_cls, ft);
+}
+
 void launch_halo_wait(const unsigned long long* flags, int nb0, int nb1, cudaStream_t s) {
   halo_wait_kernel<<<1, 1, 0, s>>>(flags, nb0, nb1);
 }
@@ -1157,6 +1166,7 @@ void preload_kernels() {
   preload_variant<27, LBM_KBC, double>();
   cudaFuncAttributes a;
   cudaFuncGetAttributes(&a, halo_wait_kernel);
+  cudaFuncGetAttributes(&a, bc_update_kernel);
   cudaFuncGetAttributes(&a, coalesce_kernel<float>);
   cudaFuncGetAttributes(&a, probe_kernel<19, float>);
   cudaFuncGetAttributes(&a, vavg_gather<19, float>);
