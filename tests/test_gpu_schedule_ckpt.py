@@ -154,3 +154,33 @@ def test_checkpoint_partitioned_bitwise():
     got = [pg2.macroscopic(L) for L in range(prob.levels)]
     pg2.close()
     _same(ref, got)
+
+
+@pytest.mark.parametrize("prec", [0, 1])
+def test_set_bc_mid_run_applies_from_next_step(prec):
+    """lbm_set_bc is enqueued on the grid's stream (include/lbmr.h): a lid
+    change after 2 coarse steps acts on steps 3.. only, i.e. equals a grid
+    built with the new lid that resumes from the 2-step checkpoint."""
+    import dataclasses
+    lbmr = _lbmr()
+    prob = I.cavity2("r")
+    u2 = (0.03, 0.0, 0.01)
+    prob2 = dataclasses.replace(prob, bc={**prob.bc, I.CLS_LID: (I.BC_VELOCITY, u2)})
+    g = lbmr.grid_from_problem(prob, precision=prec)
+    g.step(2)
+    g.set_bc(I.CLS_LID, lbmr.BC_VELOCITY, u2)
+    g.step(3)
+    changed = _fields(g, prob.levels)
+    g.close()
+    h = lbmr.grid_from_problem(prob, precision=prec)
+    h.step(2)
+    ck = h.save_checkpoint()
+    h.step(3)
+    unchanged = _fields(h, prob.levels)
+    h.close()
+    k = lbmr.grid_from_problem(prob2, precision=prec, init=False)
+    k.load_checkpoint(ck)
+    k.step(3)
+    _same(changed, _fields(k, prob.levels))
+    k.close()
+    assert not np.array_equal(np.nan_to_num(changed[0][1]), np.nan_to_num(unchanged[0][1]))
