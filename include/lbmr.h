@@ -146,7 +146,11 @@ lbm_status lbm_probe(lbm_grid* g, int32_t level, int64_t n, const int64_t* xyz, 
  * Synchronises. */
 lbm_status lbm_stats(lbm_grid* g, int64_t* leaves_per_level, double* total_mass);
 
-/* Grid description and sizes (no device work). */
+/* Grid description and sizes (no device work).  launches_per_step counts every
+ * kernel one coarse step launches (level kernels, coalescence gathers, the
+ * halo waits of a partitioned grid); device_bytes equals what
+ * lbm_grid_analyze predicts for the same desc/masks (scratch buffers of the
+ * diagnostics calls, allocated on demand, are not included). */
 lbm_status lbm_grid_get_info(const lbm_grid* g, lbm_grid_info* info);
 
 /* Instrumented run for measurement: advances n_coarse steps launching the
@@ -193,7 +197,11 @@ lbm_status lbm_checkpoint_load(lbm_grid* g, const void* host, int64_t size);
 /* Block until all work enqueued on the grid's stream is done. */
 lbm_status lbm_synchronize(lbm_grid* g);
 
-/* Destroy the grid and free its device memory; NULL is a no-op. */
+/* Destroy the grid and free its device memory; NULL is a no-op.  Waits for the
+ * grid's own stream only: on a partitioned grid the neighbours' kernels store
+ * into this grid's buffers, so every rank must synchronise its grid and pass a
+ * barrier before any rank destroys its grid (PartitionedGrid.close does this
+ * for grids of one process). */
 void lbm_grid_destroy(lbm_grid* g);
 
 /* Thread-local text of the last non-OK status ("" if none). */
@@ -206,8 +214,8 @@ const char* lbm_version(void);
 
 /* Validate masks and build the block tables on the host only, filling the
  * counts of `info` (levels, Q, leaves, blocks, special blocks/cells,
- * kernels_per_step); device_bytes is the population + table footprint the
- * grid would allocate.  Same validation and error codes as lbm_grid_create. */
+ * kernels_per_step); device_bytes is the population + table footprint
+ * lbm_grid_create allocates (the same allocation list).  Same validation and error codes as lbm_grid_create. */
 lbm_status lbm_grid_analyze(const lbm_grid_desc* desc, int32_t levels, const uint8_t* const* masks,
                             lbm_grid_info* info);
 
@@ -257,6 +265,13 @@ lbm_status lbm_halo_connect(lbm_grid* g, int32_t side, const void* blob, int64_t
 /* Connect `side` to a neighbour grid of this process (same device or a
  * peer-accessible one). */
 lbm_status lbm_halo_connect_local(lbm_grid* g, int32_t side, lbm_grid* peer);
+
+/* Debugging aid: the four halo-protocol counters of a partitioned grid
+ * (out[4]: [0]/[1] bumped by the -x/+x neighbour per finished kernel, [2]
+ * kernels finished by this rank, [3] protocol CTAs of the running kernel),
+ * read on a separate stream without waiting for the grid's stream.
+ * LBM_E_STATE on a single-rank grid. */
+lbm_status lbm_debug_flags(lbm_grid* g, unsigned long long* out);
 
 /* Host-only plan of one side/level of rank desc->rank: global coordinates
  * (x, y, z) of the cells it sends (its first owned layer at the cut) and of

@@ -36,8 +36,12 @@ def build(force: bool = False) -> str:
 def _load():
     global _lib
     if _lib is None:
-        build()
-        lib = ctypes.CDLL(_LIB)
+        # ORACLE_LIB: a separately built copy (tools/mutation_test.py loads
+        # deliberately mutated oracles to show that the pins catch them)
+        path = os.environ.get("ORACLE_LIB")
+        if not path:
+            path = build()
+        lib = ctypes.CDLL(path)
         P = ctypes.c_void_p
         dp = ctypes.POINTER(ctypes.c_double)
         ip = ctypes.POINTER(ctypes.c_int)

@@ -18,10 +18,12 @@
 #include <unistd.h>
 
 #include <algorithm>
+#include <bitset>
 #include <cmath>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include <string>
 #include <vector>
 
@@ -89,6 +91,7 @@ struct lbm_grid {
   uint8_t* face_dev = nullptr;
   cudaStream_t stream = nullptr;
   bool own_stream = false;
+  int device = 0;            // CUDA device the grid lives on (set by every call, restored after)
   cudaGraphExec_t graph[2] = {nullptr, nullptr};
   bool needs_prologue = true;
   bool init_locked = false;  // a step ran since the last init_uniform
@@ -115,6 +118,21 @@ struct lbm_grid {
 };
 
 namespace {
+
+// Every call on a grid runs on the grid's device and restores the caller's
+// current device afterwards (grids of one process may live on
+// different devices).
+struct DeviceGuard {
+  int prev = -1;
+  bool switched = false;
+  explicit DeviceGuard(const lbm_grid* g) {
+    if (g && cudaGetDevice(&prev) == cudaSuccess && prev != g->device)
+      switched = cudaSetDevice(g->device) == cudaSuccess;
+  }
+  ~DeviceGuard() {
+    if (switched) cudaSetDevice(prev);
+  }
+};
 
 template <typename T>
 lbm_status dev_upload(lbm_grid* g, T** dst, const std::vector<T>& src) {
@@ -516,15 +534,35 @@ static lbm_status build_host(const lbm_grid_desc* d, int32_t levels, const uint8
   return LBM_OK;
 }
 
-static void fill_info(const std::vector<HostLevel>& host, int Q, int prec, lbm_grid_info* info) {
+// Device bytes lbm_grid_create allocates for these host tables: the same list
+// (and the same minimum sizes) as its dev_upload / dev_alloc calls.
+static int64_t planned_device_bytes(const std::vector<HostLevel>& host, int Q, size_t ts, int n_ranks) {
+  auto up = [](size_t n, size_t es) { return (int64_t)std::max(n * es, es); };
+  auto al = [](size_t b) { return (int64_t)std::max<size_t>(b, 16); };
+  int64_t t = 0;
+  for (const HostLevel& H : host)
+    t += up(H.blkmap.size(), 4) + up(H.types.size(), 1) + up(H.origin.size(), 4) + up(H.nbr.size(), 4) +
+         up(H.special_slot.size(), 4) + up(H.cellinfo.size(), 4) + up(H.bmask.size(), 4) + up(H.links.size(), 4) +
+         up(H.coal.size(), 4) + up(H.bpeer.size(), 4) + up(H.ghost_fill.size(), 4) + up(H.coal_fill.size(), 4) +
+         up(H.coal_cand.size(), 4) + up(H.vfill.size(), 4) + up(H.vavg.size(), 4) + al((H.vavg.size() / 36) * ts) +
+         2 * al((size_t)H.nfluid * Q * kCells * ts);
+  if (n_ranks > 1) t += al(4 * sizeof(unsigned long long));
+  t += al(sizeof(BCEntry) * 256) + al(32);
+  return t;
+}
+
+static void fill_info(const std::vector<HostLevel>& host, int Q, int prec, int n_ranks, lbm_grid_info* info) {
   std::memset(info, 0, sizeof(*info));
   info->levels = (int32_t)host.size();
   info->Q = Q;
   info->precision = prec;
   info->kernels_per_step = (1 << host.size()) - 1;
   info->launches_per_step = info->kernels_per_step;
+  // partitioned grid: a one-thread halo wait before every level kernel
+  if (n_ranks > 1) info->launches_per_step += info->kernels_per_step;
   for (size_t L = 0; L < host.size(); ++L) {
-    if (!host[L].coal_fill.empty()) info->launches_per_step += (int64_t)1 << L;
+    // the coalescence gather before every F_L^k (and its own halo wait when partitioned)
+    if (!host[L].coal_fill.empty()) info->launches_per_step += ((int64_t)1 << L) * (n_ranks > 1 ? 2 : 1);
     if (!host[L].vavg.empty()) info->launches_per_step += (int64_t)2 << L;
     info->leaves[L] = host[L].leaves;
     info->blocks[L] = host[L].nfluid;
@@ -550,14 +588,8 @@ lbm_status lbm_grid_analyze(const lbm_grid_desc* d, int32_t levels, const uint8_
   } else if ((s = build_host(d, levels, masks, host))) {
     return s;
   }
-  fill_info(host, d->lattice, d->precision, info);
-  const int64_t ts = d->precision == LBM_FP32 ? 4 : 8;
-  int64_t bytes = 0;
-  for (const HostLevel& H : host)
-    bytes += 2 * (int64_t)H.nfluid * d->lattice * kCells * ts + (int64_t)H.blkmap.size() * 4 +
-             (int64_t)H.types.size() + (int64_t)H.nbr.size() * 4 + (int64_t)H.cellinfo.size() * 4 +
-             (int64_t)H.links.size() * 4 + (int64_t)H.coal.size() * 4 + (int64_t)H.origin.size() * 4;
-  info->device_bytes = bytes;
+  fill_info(host, d->lattice, d->precision, d->n_ranks, info);
+  info->device_bytes = planned_device_bytes(host, d->lattice, d->precision == LBM_FP32 ? 4 : 8, d->n_ranks);
   return LBM_OK;
 }
 
@@ -606,6 +638,10 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     g_err = keep;
     return s;
   };
+  if (cudaGetDevice(&g->device) != cudaSuccess) {
+    delete g;
+    return fail(LBM_E_CUDA, "cudaGetDevice failed (no CUDA device?)");
+  }
   if (d->stream) {
     g->stream = static_cast<cudaStream_t>(d->stream);
   } else {
@@ -616,10 +652,16 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     g->own_stream = true;
   }
 
-  static bool preloaded = false;
-  if (!preloaded) {
-    preload_kernels();
-    preloaded = true;
+  // eager kernel loading, once per device (the function attributes and the
+  // module load are per device; guarded for grids created from several threads)
+  {
+    static std::mutex mu;
+    static std::bitset<64> preloaded;
+    std::lock_guard<std::mutex> lock(mu);
+    if (g->device >= 0 && g->device < 64 && !preloaded[g->device]) {
+      preload_kernels();
+      preloaded[g->device] = true;
+    }
   }
   g->dev.resize(levels);
   lbm_status s;
@@ -687,6 +729,7 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
 lbm_status lbm_set_bc(lbm_grid* g, int32_t cls, int32_t kind, const double* u) {
   g_err.clear();
   if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  DeviceGuard dg_(g);
   if (cls < 2 || cls > 254) return fail(LBM_E_INVAL, "bc_class must be in 2..254");
   if (kind != LBM_BC_NOSLIP && kind != LBM_BC_VELOCITY && kind != LBM_BC_OUTFLOW)
     return fail(LBM_E_INVAL, "bad BC kind");
@@ -700,44 +743,59 @@ lbm_status lbm_set_bc(lbm_grid* g, int32_t cls, int32_t kind, const double* u) {
   return LBM_OK;
 }
 
+// Host -> device traffic of the init / output calls goes through the grid's
+// reusable pinned host and device scratch (no allocation per call), in chunks
+// of kIoChunkBlocks blocks so the scratch stays small (64 MiB) at any size.
+constexpr int32_t kIoChunkBlocks = 4096;
+
 static lbm_status init_level(lbm_grid* g, int L, const double* rho, const double* u, double rho0, const double* u0) {
   const HostLevel& H = g->host[L];
-  const size_t ncell = (size_t)H.nfluid * kCells;
-  std::vector<double> r(ncell, rho0), v(ncell * 3, 0.0);
-  if (u0)
-    for (size_t c = 0; c < ncell; ++c) { v[3 * c] = u0[0]; v[3 * c + 1] = u0[1]; v[3 * c + 2] = u0[2]; }
-  if (rho || u) {
+  const size_t chunk_cells = (size_t)kIoChunkBlocks * kCells;
+  void *dv = nullptr, *hv = nullptr;
+  lbm_status st;
+  CUDA_TRY(cudaStreamSynchronize(g->stream));  // queued work may still read the scratch
+  if ((st = scratch_dev(g, chunk_cells * 4 * sizeof(double), &dv)) ||
+      (st = scratch_host(g, chunk_cells * 4 * sizeof(double), &hv)))
+    return st;
+  for (int32_t b0 = 0; b0 < H.nfluid; b0 += kIoChunkBlocks) {
+    const int32_t nb = std::min(kIoChunkBlocks, H.nfluid - b0);
+    const size_t ncell = (size_t)nb * kCells;
+    // chunk layout: rho[ncell] then u[3 ncell]
+    double* r = static_cast<double*>(hv);
+    double* v = r + ncell;
 #pragma omp parallel for schedule(static)
-    for (int32_t b = 0; b < H.nfluid; ++b) {
+    for (int32_t i = 0; i < nb; ++i) {
+      const int32_t b = b0 + i;
       const int64_t ox = (int64_t)H.origin[3 * b] * kBlock, oy = (int64_t)H.origin[3 * b + 1] * kBlock,
                     oz = (int64_t)H.origin[3 * b + 2] * kBlock;
       for (int l = 0; l < kCells; ++l) {
-        if (H.types[(size_t)b * kCells + l] != kFluid) continue;
+        const size_t k = (size_t)i * kCells + l;
+        r[k] = rho0;
+        v[3 * k] = u0 ? u0[0] : 0.0;
+        v[3 * k + 1] = u0 ? u0[1] : 0.0;
+        v[3 * k + 2] = u0 ? u0[2] : 0.0;
+        if (!(rho || u) || H.types[(size_t)b * kCells + l] != kFluid) continue;
         const int64_t x = ox + (l & 7), y = oy + ((l >> 3) & 7), z = oz + (l >> 6);
         if (x < H.owned_lo || x >= H.owned_hi) continue;  // halo cells come from the neighbour
         const int64_t c = ((x - H.owned_lo) * H.n[1] + y) * H.n[2] + z;
-        const size_t k = (size_t)b * kCells + l;
         if (rho) r[k] = rho[c];
         if (u) { v[3 * k] = u[3 * c]; v[3 * k + 1] = u[3 * c + 1]; v[3 * k + 2] = u[3 * c + 2]; }
       }
     }
+    double* dr = static_cast<double*>(dv);
+    CUDA_TRY(cudaMemcpyAsync(dr, r, ncell * 4 * sizeof(double), cudaMemcpyHostToDevice, g->stream));
+    launch_init_eq(g->Q, g->prec, static_cast<char*>(g->dev[L].pop[0]) + (size_t)b0 * g->Q * kCells * g->tsize,
+                   g->dev[L].types + (size_t)b0 * kCells, nb, dr, dr + ncell, g->stream);
+    CUDA_TRY(cudaGetLastError());
+    CUDA_TRY(cudaStreamSynchronize(g->stream));  // the pinned chunk is refilled next
   }
-  double *dr = nullptr, *du = nullptr;
-  CUDA_TRY(cudaMalloc(&dr, std::max<size_t>(ncell, 1) * sizeof(double)));
-  CUDA_TRY(cudaMalloc(&du, std::max<size_t>(ncell, 1) * 3 * sizeof(double)));
-  CUDA_TRY(cudaMemcpyAsync(dr, r.data(), ncell * sizeof(double), cudaMemcpyHostToDevice, g->stream));
-  CUDA_TRY(cudaMemcpyAsync(du, v.data(), ncell * 3 * sizeof(double), cudaMemcpyHostToDevice, g->stream));
-  launch_init_eq(g->Q, g->prec, g->dev[L].pop[0], g->dev[L].types, H.nfluid, dr, du, g->stream);
-  CUDA_TRY(cudaGetLastError());
-  CUDA_TRY(cudaStreamSynchronize(g->stream));
-  cudaFree(dr);
-  cudaFree(du);
   return LBM_OK;
 }
 
 lbm_status lbm_init_equilibrium(lbm_grid* g, int32_t level, const double* rho, const double* u) {
   g_err.clear();
   if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  DeviceGuard dg_(g);
   if (g->broken) return fail(LBM_E_STATE, "grid is in an error state");
   if (level < 0 || level >= g->levels) return fail(LBM_E_INVAL, "level out of range");
   if (g->init_locked)
@@ -752,6 +810,7 @@ lbm_status lbm_init_equilibrium(lbm_grid* g, int32_t level, const double* rho, c
 lbm_status lbm_init_uniform(lbm_grid* g, double rho0, const double* u0) {
   g_err.clear();
   if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  DeviceGuard dg_(g);
   if (g->broken) return fail(LBM_E_STATE, "grid is in an error state");
   for (int L = 0; L < g->levels; ++L) {
     lbm_status s = init_level(g, L, nullptr, nullptr, rho0, u0);
@@ -766,6 +825,7 @@ lbm_status lbm_init_uniform(lbm_grid* g, double rho0, const double* u0) {
 lbm_status lbm_step(lbm_grid* g, int32_t n) {
   g_err.clear();
   if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  DeviceGuard dg_(g);
   if (g->broken) return fail(LBM_E_STATE, "grid is in an error state");
   if (n < 0) return fail(LBM_E_INVAL, "n_coarse must be >= 0");
   if (n == 0) return LBM_OK;
@@ -801,6 +861,7 @@ lbm_status lbm_step(lbm_grid* g, int32_t n) {
 lbm_status lbm_set_schedule(lbm_grid* g, int32_t mode) {
   g_err.clear();
   if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  DeviceGuard dg_(g);
   if (mode < 0 || mode > (LBM_SCHED_UNFUSED | LBM_SCHED_NO_GRAPH)) return fail(LBM_E_INVAL, "bad schedule mode");
   if ((mode & LBM_SCHED_UNFUSED) && g->n_ranks > 1)
     return fail(LBM_E_UNSUPPORTED, "the unfused schedule is single-rank only");
@@ -845,6 +906,7 @@ lbm_status lbm_checkpoint_size(const lbm_grid* g, int64_t* bytes) {
 lbm_status lbm_checkpoint_save(lbm_grid* g, void* host, int64_t capacity) {
   g_err.clear();
   if (!g || !host) return fail(LBM_E_INVAL, "NULL argument");
+  DeviceGuard dg_(g);
   if (g->broken) return fail(LBM_E_STATE, "grid is in an error state");
   int64_t need = 0;
   lbm_checkpoint_size(g, &need);
@@ -869,6 +931,11 @@ lbm_status lbm_checkpoint_save(lbm_grid* g, void* host, int64_t capacity) {
   char* out = static_cast<char*>(host);
   std::memcpy(out, &h, sizeof(h));
   int64_t off = sizeof(h);
+  // partitioned grid: the buffers include halo cells the neighbours' last
+  // kernels store into; wait (on the device) until every neighbour has
+  // finished the cut-plane part of all kernels this rank has run
+  if (g->n_ranks > 1 && !g->needs_prologue) launch_halo_wait(g->flags, g->has_nb[0], g->has_nb[1], g->stream);
+  CUDA_TRY(cudaGetLastError());
   CUDA_TRY(cudaStreamSynchronize(g->stream));
   for (int L = 0; L < g->levels; ++L) {
     const size_t b = pop_bytes(g, L);
@@ -882,6 +949,7 @@ lbm_status lbm_checkpoint_save(lbm_grid* g, void* host, int64_t capacity) {
 lbm_status lbm_checkpoint_load(lbm_grid* g, const void* host, int64_t size) {
   g_err.clear();
   if (!g || !host) return fail(LBM_E_INVAL, "NULL argument");
+  DeviceGuard dg_(g);
   if (g->broken) return fail(LBM_E_STATE, "grid is in an error state");
   if (size < (int64_t)sizeof(CkptHeader)) return fail(LBM_E_INVAL, "checkpoint too small");
   CkptHeader h;
@@ -914,6 +982,7 @@ lbm_status lbm_checkpoint_load(lbm_grid* g, const void* host, int64_t size) {
 lbm_status lbm_profile_levels(lbm_grid* g, int32_t n, double* ms_per_level, int64_t* launches_per_level) {
   g_err.clear();
   if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  DeviceGuard dg_(g);
   if (g->broken) return fail(LBM_E_STATE, "grid is in an error state");
   for (int sd = 0; sd < 2; ++sd)
     if (g->n_ranks > 1 && g->has_nb[sd] && !g->connected[sd])
@@ -960,6 +1029,7 @@ lbm_status lbm_profile_levels(lbm_grid* g, int32_t n, double* ms_per_level, int6
 lbm_status lbm_synchronize(lbm_grid* g) {
   g_err.clear();
   if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  DeviceGuard dg_(g);
   CUDA_TRY(cudaStreamSynchronize(g->stream));
   return LBM_OK;
 }
@@ -967,39 +1037,47 @@ lbm_status lbm_synchronize(lbm_grid* g) {
 lbm_status lbm_macroscopic(lbm_grid* g, int32_t L, double* rho, double* u) {
   g_err.clear();
   if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  DeviceGuard dg_(g);
   if (L < 0 || L >= g->levels) return fail(LBM_E_INVAL, "level out of range");
   const HostLevel& H = g->host[L];
-  const size_t ncell = (size_t)H.nlaunch * kCells;
-  double *dr = nullptr, *du = nullptr;
-  CUDA_TRY(cudaStreamSynchronize(g->stream));
-  CUDA_TRY(cudaMalloc(&dr, std::max<size_t>(ncell, 1) * sizeof(double)));
-  CUDA_TRY(cudaMalloc(&du, std::max<size_t>(ncell, 1) * 3 * sizeof(double)));
-  launch_macroscopic(g->Q, g->prec, g->dev[L].pop[cur_buf(g, L)], g->dev[L].nbr, H.nlaunch, dr, du, nullptr,
-                     g->stream);
-  std::vector<double> r(ncell), v(3 * ncell);
-  CUDA_TRY(cudaGetLastError());
-  CUDA_TRY(cudaMemcpyAsync(r.data(), dr, ncell * sizeof(double), cudaMemcpyDeviceToHost, g->stream));
-  CUDA_TRY(cudaMemcpyAsync(v.data(), du, 3 * ncell * sizeof(double), cudaMemcpyDeviceToHost, g->stream));
-  CUDA_TRY(cudaStreamSynchronize(g->stream));
-  cudaFree(dr);
-  cudaFree(du);
   // dense arrays over the owned slab of this rank (the whole level on one rank)
   const int64_t N = (H.owned_hi - H.owned_lo) * H.n[1] * H.n[2];
   const double nan = std::nan("");
   if (rho) std::fill(rho, rho + N, nan);
   if (u) std::fill(u, u + 3 * N, nan);
+  const size_t chunk_cells = (size_t)kIoChunkBlocks * kCells;
+  void *dv = nullptr, *hv = nullptr;
+  lbm_status st;
+  CUDA_TRY(cudaStreamSynchronize(g->stream));
+  if ((st = scratch_dev(g, chunk_cells * 4 * sizeof(double), &dv)) ||
+      (st = scratch_host(g, chunk_cells * 4 * sizeof(double), &hv)))
+    return st;
+  const char* pop = static_cast<const char*>(g->dev[L].pop[cur_buf(g, L)]);
+  for (int32_t b0 = 0; b0 < H.nlaunch; b0 += kIoChunkBlocks) {
+    const int32_t nb = std::min(kIoChunkBlocks, H.nlaunch - b0);
+    const size_t ncell = (size_t)nb * kCells;
+    double* dr = static_cast<double*>(dv);
+    launch_macroscopic(g->Q, g->prec, pop + (size_t)b0 * g->Q * kCells * g->tsize, g->dev[L].nbr + (size_t)b0 * kRec,
+                       nb, dr, dr + ncell, nullptr, g->stream);
+    CUDA_TRY(cudaGetLastError());
+    CUDA_TRY(cudaMemcpyAsync(hv, dr, ncell * 4 * sizeof(double), cudaMemcpyDeviceToHost, g->stream));
+    CUDA_TRY(cudaStreamSynchronize(g->stream));
+    const double* r = static_cast<const double*>(hv);
+    const double* v = r + ncell;
 #pragma omp parallel for schedule(static)
-  for (int32_t b = 0; b < H.nlaunch; ++b) {
-    const int64_t ox = (int64_t)H.origin[3 * b] * kBlock, oy = (int64_t)H.origin[3 * b + 1] * kBlock,
-                  oz = (int64_t)H.origin[3 * b + 2] * kBlock;
-    for (int l = 0; l < kCells; ++l) {
-      if (H.types[(size_t)b * kCells + l] != kFluid) continue;
-      const int64_t x = ox + (l & 7), y = oy + ((l >> 3) & 7), z = oz + (l >> 6);
-      if (x < H.owned_lo || x >= H.owned_hi) continue;
-      const int64_t c = ((x - H.owned_lo) * H.n[1] + y) * H.n[2] + z;
-      const size_t k = (size_t)b * kCells + l;
-      if (rho) rho[c] = r[k];
-      if (u) { u[3 * c] = v[3 * k]; u[3 * c + 1] = v[3 * k + 1]; u[3 * c + 2] = v[3 * k + 2]; }
+    for (int32_t i = 0; i < nb; ++i) {
+      const int32_t b = b0 + i;
+      const int64_t ox = (int64_t)H.origin[3 * b] * kBlock, oy = (int64_t)H.origin[3 * b + 1] * kBlock,
+                    oz = (int64_t)H.origin[3 * b + 2] * kBlock;
+      for (int l = 0; l < kCells; ++l) {
+        if (H.types[(size_t)b * kCells + l] != kFluid) continue;
+        const int64_t x = ox + (l & 7), y = oy + ((l >> 3) & 7), z = oz + (l >> 6);
+        if (x < H.owned_lo || x >= H.owned_hi) continue;
+        const int64_t c = ((x - H.owned_lo) * H.n[1] + y) * H.n[2] + z;
+        const size_t k = (size_t)i * kCells + l;
+        if (rho) rho[c] = r[k];
+        if (u) { u[3 * c] = v[3 * k]; u[3 * c + 1] = v[3 * k + 1]; u[3 * c + 2] = v[3 * k + 2]; }
+      }
     }
   }
   return LBM_OK;
@@ -1008,6 +1086,7 @@ lbm_status lbm_macroscopic(lbm_grid* g, int32_t L, double* rho, double* u) {
 lbm_status lbm_probe(lbm_grid* g, int32_t L, int64_t n, const int64_t* xyz, double* rho, double* u) {
   g_err.clear();
   if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  DeviceGuard dg_(g);
   if (L < 0 || L >= g->levels) return fail(LBM_E_INVAL, "level out of range");
   if (n < 0 || (n > 0 && (!xyz || !rho || !u))) return fail(LBM_E_INVAL, "bad probe arguments");
   if (n == 0) return LBM_OK;
@@ -1053,6 +1132,7 @@ lbm_status lbm_probe(lbm_grid* g, int32_t L, int64_t n, const int64_t* xyz, doub
 lbm_status lbm_stats(lbm_grid* g, int64_t* leaves, double* mass) {
   g_err.clear();
   if (!g) return fail(LBM_E_INVAL, "NULL grid");
+  DeviceGuard dg_(g);
   if (leaves)
     for (int L = 0; L < g->levels; ++L) leaves[L] = g->host[L].leaves;
   if (!mass) return LBM_OK;
@@ -1090,7 +1170,7 @@ lbm_status lbm_stats(lbm_grid* g, int64_t* leaves, double* mass) {
 lbm_status lbm_grid_get_info(const lbm_grid* g, lbm_grid_info* info) {
   g_err.clear();
   if (!g || !info) return fail(LBM_E_INVAL, "NULL argument");
-  fill_info(g->host, g->Q, g->prec, info);
+  fill_info(g->host, g->Q, g->prec, g->n_ranks, info);
   info->device_bytes = g->device_bytes;
   info->steps_done = g->steps;
   return LBM_OK;
@@ -1156,6 +1236,7 @@ lbm_status open_ipc(lbm_grid* g, const cudaIpcMemHandle_t& h, void** out) {
 lbm_status lbm_halo_export(const lbm_grid* g, int32_t side, void* blob, int64_t capacity, int64_t* size) {
   g_err.clear();
   if (!g || side < 0 || side > 1) return fail(LBM_E_INVAL, "bad arguments");
+  DeviceGuard dg_(g);
   if (g->n_ranks < 2 || !g->has_nb[side]) return fail(LBM_E_STATE, "no neighbour on this side");
   int64_t need = sizeof(HaloBlob);
   for (int L = 0; L < g->levels; ++L) need += (int64_t)g->host[L].halo[side].size() * 4;
@@ -1202,6 +1283,7 @@ static lbm_status check_counts(lbm_grid* g, int side, const int64_t* count) {
 lbm_status lbm_halo_connect(lbm_grid* g, int32_t side, const void* blob, int64_t size) {
   g_err.clear();
   if (!g || !blob || side < 0 || side > 1) return fail(LBM_E_INVAL, "bad arguments");
+  DeviceGuard dg_(g);
   if (g->n_ranks < 2 || !g->has_nb[side]) return fail(LBM_E_STATE, "no neighbour on this side");
   if (size < (int64_t)sizeof(HaloBlob)) return fail(LBM_E_INVAL, "blob too small");
   HaloBlob h;
@@ -1239,6 +1321,7 @@ lbm_status lbm_halo_connect(lbm_grid* g, int32_t side, const void* blob, int64_t
 lbm_status lbm_halo_connect_local(lbm_grid* g, int32_t side, lbm_grid* peer) {
   g_err.clear();
   if (!g || !peer || side < 0 || side > 1) return fail(LBM_E_INVAL, "bad arguments");
+  DeviceGuard dg_(g);
   if (g->n_ranks < 2 || !g->has_nb[side] || !peer->has_nb[1 - side]) return fail(LBM_E_STATE, "no neighbour");
   if (peer->levels != g->levels || peer->Q != g->Q || peer->prec != g->prec || peer->n_ranks != g->n_ranks)
     return fail(LBM_E_COMM, "peer grid does not match");
@@ -1246,6 +1329,17 @@ lbm_status lbm_halo_connect_local(lbm_grid* g, int32_t side, lbm_grid* peer) {
   for (int L = 0; L < g->levels; ++L) count[L] = (int64_t)peer->host[L].halo[1 - side].size();
   lbm_status s = check_counts(g, side, count);
   if (s) return s;
+  if (peer->device != g->device) {
+    // the level kernels store into the peer's buffers and bump its flags:
+    // direct peer access over NVLink from this grid's device
+    int ok = 0;
+    CUDA_TRY(cudaDeviceCanAccessPeer(&ok, g->device, peer->device));
+    if (!ok) return fail(LBM_E_COMM, "devices " + std::to_string(g->device) + " and " + std::to_string(peer->device) +
+                                         " have no peer access");
+    cudaError_t e = cudaDeviceEnablePeerAccess(peer->device, 0);
+    if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
+    else if (e != cudaSuccess) return fail(LBM_E_COMM, std::string("cudaDeviceEnablePeerAccess: ") + cudaGetErrorString(e));
+  }
   if ((s = invalidate_graphs(g))) return s;
   for (int L = 0; L < g->levels; ++L) {
     DevLevel& D = g->dev[L];
@@ -1292,9 +1386,12 @@ lbm_status lbm_halo_plan(const lbm_grid_desc* d, int32_t levels, const uint8_t* 
   return LBM_OK;
 }
 
-// debugging aid (not in the public header): the four halo-protocol counters
-extern "C" lbm_status lbm_debug_flags(lbm_grid* g, unsigned long long* out) {
-  if (!g || !g->flags) return fail(LBM_E_STATE, "no flags");
+// the four halo-protocol counters (declared in lbmr.h as a debugging aid)
+lbm_status lbm_debug_flags(lbm_grid* g, unsigned long long* out) {
+  g_err.clear();
+  if (!g || !out) return fail(LBM_E_INVAL, "NULL argument");
+  if (!g->flags) return fail(LBM_E_STATE, "not a partitioned grid (no halo-protocol flags)");
+  DeviceGuard dg_(g);
   cudaStream_t s;
   CUDA_TRY(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
   CUDA_TRY(cudaMemcpyAsync(out, g->flags, 4 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
@@ -1305,6 +1402,7 @@ extern "C" lbm_status lbm_debug_flags(lbm_grid* g, unsigned long long* out) {
 
 void lbm_grid_destroy(lbm_grid* g) {
   if (!g) return;
+  DeviceGuard dg_(g);
   if (g->stream) cudaStreamSynchronize(g->stream);
   for (int p = 0; p < 2; ++p)
     if (g->graph[p]) cudaGraphExecDestroy(g->graph[p]);

@@ -837,12 +837,33 @@ __global__ void __launch_bounds__(StepCta<Q, COLL, T>::threads, StepCta<Q, COLL,
 // all kernels this rank has completed (its bumps of our flag reach our
 // kernel count).  A separate one-CTA launch, so that no CTA of a level kernel
 // ever spins: partitions emulated on one device cannot starve each other.
+// The spin is bounded: a neighbour that never arrives (a rank that died or
+// stopped stepping) turns into a device trap after kHaloWaitTimeoutNs instead
+// of a hung GPU, so the caller's next synchronising call reports LBM_E_CUDA.
+#ifndef LBMR_HALO_WAIT_TIMEOUT_S
+#define LBMR_HALO_WAIT_TIMEOUT_S 120
+#endif
+constexpr unsigned long long kHaloWaitTimeoutNs = (unsigned long long)LBMR_HALO_WAIT_TIMEOUT_S * 1000000000ull;
+
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+
 __global__ void halo_wait_kernel(const unsigned long long* flags, int nb0, int nb1) {
   const unsigned long long mine = *(volatile const unsigned long long*)(flags + 2);
-  if (nb0)
-    while (ld_acquire_sys(flags + 0) < mine) __nanosleep(256);
-  if (nb1)
-    while (ld_acquire_sys(flags + 1) < mine) __nanosleep(256);
+  const unsigned long long t0 = globaltimer_ns();
+  for (int s = 0; s < 2; ++s) {
+    if (!(s == 0 ? nb0 : nb1)) continue;
+    while (ld_acquire_sys(flags + s) < mine) {
+      __nanosleep(256);
+      if (globaltimer_ns() - t0 > kHaloWaitTimeoutNs) {
+        printf("lbmr: halo wait timed out (side %d: %llu of %llu kernels)\n", s, ld_acquire_sys(flags + s), mine);
+        __trap();
+      }
+    }
+  }
 }
 
 template <int Q, int COLL, typename T, bool STREAM>

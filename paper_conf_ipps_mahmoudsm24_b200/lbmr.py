@@ -62,7 +62,7 @@ EXPORTS = ["lbm_grid_create", "lbm_set_bc", "lbm_init_equilibrium", "lbm_init_un
            "lbm_grid_destroy", "lbm_last_error", "lbm_version", "lbm_grid_analyze", "lbm_schedule",
            "lbm_lattice_table", "lbm_omega_level", "lbm_partition_cuts", "lbm_grid_slab", "lbm_halo_export",
            "lbm_halo_connect", "lbm_halo_connect_local", "lbm_halo_plan", "lbm_set_schedule",
-           "lbm_checkpoint_size", "lbm_checkpoint_save", "lbm_checkpoint_load", "lbm_probe"]
+           "lbm_checkpoint_size", "lbm_checkpoint_save", "lbm_checkpoint_load", "lbm_probe", "lbm_debug_flags"]
 
 _lib = None
 
@@ -113,6 +113,7 @@ def load_library(path: str = LIB_PATH):
     lib.lbm_checkpoint_size.argtypes = [P, lp]
     lib.lbm_checkpoint_save.argtypes = [P, ctypes.c_void_p, ctypes.c_int64]
     lib.lbm_checkpoint_load.argtypes = [P, ctypes.c_void_p, ctypes.c_int64]
+    lib.lbm_debug_flags.argtypes = [P, ctypes.POINTER(ctypes.c_ulonglong)]
     lib.lbm_last_error.restype = ctypes.c_char_p
     lib.lbm_version.restype = ctypes.c_char_p
     for name in EXPORTS:
@@ -370,6 +371,12 @@ class Grid:
         buf = np.ascontiguousarray(buf, dtype=np.uint8)
         _check(self.lib.lbm_checkpoint_load(self.h, buf.ctypes.data, buf.nbytes))
 
+    def debug_flags(self):
+        """Halo-protocol counters of a partitioned grid (lbm_debug_flags)."""
+        out = (ctypes.c_ulonglong * 4)()
+        _check(self.lib.lbm_debug_flags(self.h, out))
+        return [int(v) for v in out]
+
     def profile_levels(self, n_coarse: int):
         ms = np.zeros(self.levels)
         cnt = np.zeros(self.levels, dtype=np.int64)
@@ -438,6 +445,11 @@ class PartitionedGrid:
         return np.concatenate([p[0] for p in parts], axis=0), np.concatenate([p[1] for p in parts], axis=0)
 
     def close(self):
+        # every slab's last kernels may still be storing into a neighbour's
+        # buffers: wait for all of them before freeing any
+        for g in self.grids:
+            if g.h is not None:
+                g.synchronize()
         for g in self.grids:
             g.close()
 
