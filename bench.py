@@ -173,6 +173,123 @@ def cpu_baseline(prob):
             "seconds": dt}
 
 
+def lib_build_id():
+    """sha256 prefix of the liblbmr.so this run loads (labels measurements
+    taken from another process, e.g. the ncu traffic capture)."""
+    import hashlib
+    from paper_conf_ipps_mahmoudsm24_b200 import lbmr
+    with open(lbmr.LIB_PATH, "rb") as f:
+        return hashlib.sha256(f.read()).hexdigest()[:16]
+
+
+def level_profile(g, prob, prec, lbmr, profile_steps, leaves_local):
+    """Per-level device time of the level kernels (lbm_profile_step: the
+    coarse step captured into an instrumented CUDA graph with event nodes
+    around every level kernel and its coalescence gather, so no host launch
+    gaps are timed) and the roofline object of the dominant kernel.  `frac`
+    is the level kernel's own; `frac_incl_gather` charges the level with the
+    gather kernel that feeds it."""
+    ms_lvl, gather_ms, cnt_lvl = g.profile_step(profile_steps)
+    tsz = 4 if prec == lbmr.FP32 else 8
+    bpu = 2 * prob.Q * tsz
+    dom = int(np.argmax(ms_lvl))
+    per_launch_ms = ms_lvl[dom] / max(cnt_lvl[dom], 1)
+    achieved = leaves_local[dom] * bpu / (per_launch_ms * 1e-3) / 1e9
+    peak, peak_src = peak_hbm()
+    per_level = []
+    for L in range(prob.levels):
+        pl = ms_lvl[L] / max(cnt_lvl[L], 1)
+        gbs = leaves_local[L] * bpu / (pl * 1e-3) / 1e9 if pl > 0 else None
+        gl = gather_ms[L] / max(cnt_lvl[L], 1)
+        per_level.append({"level": L, "leaves": leaves_local[L], "launches": int(cnt_lvl[L]), "ms_per_launch": pl,
+                          "GBs": gbs, "frac": gbs / peak if gbs else None,
+                          "gather_ms_per_launch": gl,
+                          "frac_incl_gather": leaves_local[L] * bpu / ((pl + gl) * 1e-3) / 1e9 / peak if pl > 0 else None,
+                          "share_of_step": (ms_lvl[L] + gather_ms[L]) / max(ms_lvl.sum() + gather_ms.sum(), 1e-12)})
+    roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+            "kernel": f"level_step L{dom}", "bytes_per_update": bpu, "peak_source": peak_src,
+            "algorithmic_bytes_per_launch": leaves_local[dom] * bpu, "ms_per_launch": per_launch_ms}
+    return roof, per_level, dom
+
+
+def ncu_traffic(config, precision, levels, timeout=240):
+    """DRAM bytes (dram__bytes_read.sum + dram__bytes_write.sum) of one launch
+    of the dominant (finest-level) kernel, measured now by ncu in a child
+    process running this same workload (first finest launch of the second
+    coarse step).  None if ncu is unavailable or fails."""
+    import csv
+    import io
+    import shutil
+    ncu = shutil.which("ncu") or "/usr/local/cuda/bin/ncu"
+    if not os.path.exists(ncu):
+        return None, "ncu not found"
+    skip = (1 << levels) - 1  # level_step_all launches of the first coarse step
+    cmd = [ncu, "--metrics", "dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum",
+           "--clock-control", "none", "-k", "regex:level_step_all", "-s", str(skip), "-c", "1", "--csv",
+           sys.executable, os.path.abspath(__file__), "--traffic-child", "--config", config, "--precision", precision]
+    try:
+        r = subprocess.run(cmd, capture_output=True, text=True, timeout=timeout, cwd=ROOT)
+    except Exception as e:  # noqa: BLE001
+        return None, f"ncu failed: {e!r}"[:200]
+    vals = {}
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith('"')]
+    for row in csv.reader(io.StringIO("\n".join(lines))):
+        if len(row) > 14 and row[12] in ("dram__bytes_read.sum", "dram__bytes_write.sum", "gpu__time_duration.sum"):
+            unit = row[13]
+            scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "B": 1, "KB": 1e3, "MB": 1e6, "GB": 1e9,
+                     "nsecond": 1e-3, "usecond": 1, "msecond": 1e3, "ns": 1e-3, "us": 1, "ms": 1e3}.get(unit, 1)
+            vals[row[12]] = float(row[14].replace(",", "")) * scale
+    if "dram__bytes_read.sum" not in vals:
+        return None, ("ncu gave no metrics: " + (r.stderr or r.stdout)[-200:]).replace("\n", " ")
+    return {"dram_bytes_per_launch": vals["dram__bytes_read.sum"] + vals.get("dram__bytes_write.sum", 0.0),
+            "duration_us_under_ncu": vals.get("gpu__time_duration.sum")}, "ncu, this run (child process, same build)"
+
+
+def traffic_child(args):
+    """The workload ncu_traffic() profiles: build, prologue, two coarse steps."""
+    from paper_conf_ipps_mahmoudsm24_b200 import lbmr
+    prob = CONFIGS[args.config][0]()
+    prec = lbmr.FP32 if args.precision == "fp32" else lbmr.FP64
+    g = lbmr.grid_from_problem(prob, precision=prec)
+    g.step(2)
+    g.synchronize()
+    g.close()
+
+
+def secondary_block(name, prob, prec, lbmr, steps, warmup, profile_steps, paper_mlups=None):
+    """One more workload timed in the same run (N = 1 only): MLUPS over
+    `steps` graph replays (CUDA events), the dominant kernel's roofline and
+    per-level fractions."""
+    import torch
+    stream = torch.cuda.Stream()
+    g = lbmr.grid_from_problem(prob, precision=prec, stream=stream.cuda_stream)
+    info = g.info()
+    leaves = [int(info.leaves[L]) for L in range(prob.levels)]
+    upd = updates_per_step(leaves)
+    g.step(warmup)
+    g.synchronize()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    ev0.record(stream)
+    g.step(steps)
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    ms = ev0.elapsed_time(ev1)
+    value = upd * steps / (ms * 1e3)
+    roof, per_level, _ = level_profile(g, prob, prec, lbmr, profile_steps, leaves)
+    bpu = roof["bytes_per_update"]
+    roof["step_frac"] = value * 1e6 * bpu / 1e9 / roof["peak"]
+    g.close()
+    del g
+    out = {"workload": name, "value": value, "unit": "MLUPS", "ms_per_step": ms / steps, "steps": steps,
+           "dtype": "f32" if prec == lbmr.FP32 else "f64", "leaves": leaves, "updates_per_step": upd,
+           "roofline": roof, "per_level": per_level}
+    if paper_mlups:
+        out["paper_a100_mlups"] = paper_mlups
+        out["vs_paper_a100"] = value / paper_mlups
+    return out
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -189,7 +306,16 @@ def main():
                     help="fusion ablation (lbm_set_schedule); the default is the product schedule")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--profile-steps", type=int, default=10)
+    ap.add_argument("--no-secondary", action="store_true",
+                    help="skip the secondary blocks (cfg5 fp64, Tab. I s3 fp64 KBC) of the default run")
+    ap.add_argument("--no-ncu-traffic", action="store_true", help="skip the in-run ncu DRAM-traffic capture")
+    ap.add_argument("--traffic-child", action="store_true", help=argparse.SUPPRESS)
     args = ap.parse_args()
+    if args.traffic_child:
+        if args.precision is None:
+            args.precision = DEFAULT_PRECISION.get(args.config, "fp32")
+        traffic_child(args)
+        return
     args.warmup = max(args.warmup, 3)
     if args.precision is None:
         args.precision = DEFAULT_PRECISION.get(args.config, "fp32")
@@ -269,30 +395,10 @@ def main():
         ms = float(t.item())
     value = upd * args.steps / (ms * 1e3)  # all ranks' updates / max-over-ranks time
 
-    # per-level device time (instrumented launches, CUDA events on the same stream)
-    ms_lvl, cnt_lvl = g.profile_levels(args.profile_steps)
-    tsz = 4 if prec == lbmr.FP32 else 8
-    bpu = 2 * prob.Q * tsz
-    dom = int(np.argmax(ms_lvl))
-    per_launch_ms = ms_lvl[dom] / max(cnt_lvl[dom], 1)
-    achieved = leaves_local[dom] * bpu / (per_launch_ms * 1e-3) / 1e9
-    peak, peak_src = peak_hbm()
-    per_level = []
-    for L in range(prob.levels):
-        pl = ms_lvl[L] / max(cnt_lvl[L], 1)
-        gbs = leaves_local[L] * bpu / (pl * 1e-3) / 1e9 if pl > 0 else None
-        per_level.append({"level": L, "leaves": leaves_local[L], "launches": int(cnt_lvl[L]), "ms_per_launch": pl,
-                          "GBs": gbs, "frac": gbs / peak if gbs else None,
-                          "share_of_step": ms_lvl[L] / max(ms_lvl.sum(), 1e-12)})
-    traffic = None
-    tpath = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    if os.path.exists(tpath):
-        try:
-            tj = json.load(open(tpath)).get(f"{args.config}_{args.precision}")
-            if tj:
-                traffic = tj.get("dram_bytes_per_launch")
-        except Exception:
-            traffic = None
+    # per-level device time of the level kernels (instrumented graph, CUDA events)
+    roof, per_level, dom = level_profile(g, prob, prec, lbmr, args.profile_steps, leaves_local)
+    bpu = roof["bytes_per_update"]
+    peak = roof["peak"]
 
     # e2e through the public API with host buffers: per step an H2D BC update
     # (inlet velocity) and a D2H read of the step's result at monitoring
@@ -325,6 +431,37 @@ def main():
     gi = g.info()
     dev_bytes = int(gi.device_bytes)
     g.close()
+    del g
+    # DRAM traffic of the dominant kernel, measured by ncu in this run (N = 1)
+    traffic, traffic_src = None, "not measured (N > 1: ncu never wraps a multi-rank run)"
+    if rank == 0 and ws == 1 and not args.no_ncu_traffic:
+        t, traffic_src = ncu_traffic(args.config, args.precision, prob.levels)
+        if t:
+            traffic = t["dram_bytes_per_launch"]
+            roof["traffic_duration_us_under_ncu"] = t["duration_us_under_ncu"]
+    roof["traffic"] = traffic
+    roof["traffic_source"] = traffic_src
+    roof["traffic_over_algorithmic"] = traffic / roof["algorithmic_bytes_per_launch"] if traffic else None
+    roof["build_id"] = lib_build_id()
+    # secondary workloads of the default run (N = 1): the paper's precision on
+    # the headline config, and the paper's own Tab. I workload at its largest size
+    secondary = None
+    if rank == 0 and ws == 1 and not args.no_secondary and args.config == "tunnel4" and args.schedule == "fused" \
+            and args.variant == "paper":
+        secondary = {}
+        try:
+            secondary["tunnel4_fp64"] = secondary_block(CONFIGS["tunnel4"][1] + ", fp64", prob, lbmr.FP64, lbmr,
+                                                        max(5, args.steps // 2), 3, 4)
+        except Exception as e:  # noqa: BLE001
+            secondary["tunnel4_fp64"] = {"error": repr(e)[:300]}
+        try:
+            p3 = I.sphere_tab1(3)
+            secondary["sphere_tab1_s3_fp64"] = secondary_block(CONFIGS["sphere_tab1_s3"][1] + ", fp64 (P:L258)", p3,
+                                                               lbmr.FP64, lbmr, max(5, args.steps // 2), 3, 4,
+                                                               PAPER_MLUPS["sphere_tab1_s3"])
+            del p3
+        except Exception as e:  # noqa: BLE001
+            secondary["sphere_tab1_s3_fp64"] = {"error": repr(e)[:300]}
     cpu = None
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(prob)
@@ -344,12 +481,10 @@ def main():
                        "precision": args.precision, "schedule": args.schedule, "variant": args.variant,
                        "setup_s": round(setup_s, 2),
                        **({"paper_a100_fp64_mlups": PAPER_MLUPS[args.config]} if args.config in PAPER_MLUPS else {})},
-            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic, "kernel": f"level_step L{dom}",
-                         "bytes_per_update": bpu, "peak_source": peak_src,
-                         "step_frac": value * 1e6 / ws * bpu / 1e9 / peak,
+            "roofline": {**roof, "step_frac": value * 1e6 / ws * bpu / 1e9 / peak,
                          "note": "achieved / per_level are this rank's (rank 0) kernels" if ws > 1 else None},
             "per_level": per_level,
+            "secondary": secondary,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": launches_per_step * args.steps,

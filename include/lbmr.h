@@ -94,6 +94,8 @@ typedef struct {
   int64_t launches_per_step;         /* every kernel of one fused coarse step: the level steps plus
                                         one coalescence gather before each F_L^k whose level has
                                         coalescence ghosts                                          */
+  int32_t block_offset[16][3];       /* per level and axis: level cell c lies in 8^3 block
+                                        (c + off) >> 3 (builder-chosen alignment)     */
 } lbm_grid_info;
 
 /* Build the block-sparse multi-level grid (§V) from per-level masks.
@@ -153,27 +155,65 @@ lbm_status lbm_stats(lbm_grid* g, int64_t* leaves_per_level, double* total_mass)
  * diagnostics calls, allocated on demand, are not included). */
 lbm_status lbm_grid_get_info(const lbm_grid* g, lbm_grid_info* info);
 
-/* Instrumented run for measurement: advances n_coarse steps launching the
- * same kernels without the graph, bracketing every launch with CUDA events
- * on the grid's stream; ms_per_level[L] receives the summed device time of
- * level L's launches and launches_per_level[L] their count (either may be
- * NULL).  Synchronises. */
+/* Instrumented run for measurement: advances n_coarse steps replaying, per
+ * parity of the step index, a CUDA graph of the same launches as lbm_step's
+ * with a one-thread timestamp kernel (device global timer) before each level
+ * kernel's pre-kernels (coalescence gather / volumetric averages / ablation
+ * kernels), between them and the level kernel, and after it (eager launches
+ * instead under LBM_SCHED_NO_GRAPH).  level_ms[L]: summed
+ * device time of level L's kernels F_L^k; gather_ms[L]: of the pre-kernels
+ * feeding them; launches_per_level[L]: number of F_L^k (any may be NULL).
+ * Synchronises after every step. */
+lbm_status lbm_profile_step(lbm_grid* g, int32_t n_coarse, double* level_ms, double* gather_ms,
+                            int64_t* launches_per_level);
+
+/* lbm_profile_step with ms_per_level[L] = level_ms[L] + gather_ms[L]. */
 lbm_status lbm_profile_levels(lbm_grid* g, int32_t n_coarse, double* ms_per_level,
                               int64_t* launches_per_level);
 
-/* Kernel schedule of lbm_step / lbm_profile_levels (bit flags; default 0).
- *  LBM_SCHED_FUSED     one fused kernel F_L^k per level-substep (stream +
- *                      Explosion + Coalescence + BC + collide), 2Q values
- *                      moved per leaf — the paper's fully fused design
- *                      (Fig. 4f) in the pipelined order.
- *  LBM_SCHED_UNFUSED   ablation (Fig. 9): per level-substep a
- *                      stream-only kernel S_L^k then an in-place collision
- *                      C_L^{k+1} (4Q values per leaf).  Bitwise identical
- *                      results.  Single rank only (LBM_E_UNSUPPORTED).
- *  LBM_SCHED_NO_GRAPH  launch the kernels one by one instead of replaying
+/* Kernel schedule of lbm_step / lbm_profile_* (bit flags; default 0).  The
+ * steps of one level-substep are C (collision), A (Accumulate: fine
+ * post-collision values into the coarse-side ghost layer), S (streaming),
+ * E (Explosion) and O (Coalescence: the coarse level reads and averages the
+ * accumulated values), §IV and Fig. 4.
+ *  LBM_SCHED_FUSED     (0) one fused kernel F_L^k per level-substep (S + E +
+ *                      O + BC + C), 2Q values moved per leaf, and one small
+ *                      gather kernel before it doing A + A + O from the two
+ *                      retained fine buffers (deterministic) — the product.
+ *  LBM_SCHED_UNFUSED   (1) C and S separate: a stream-only kernel S_L^k then
+ *                      an in-place collision C_L^{k+1} (4Q values per leaf).
+ *  LBM_SCHED_NO_GRAPH  (2) launch the kernels one by one instead of replaying
  *                      the captured CUDA graph (launch-overhead ablation).
- * Takes effect at the next lbm_step; synchronises the grid's stream. */
-enum { LBM_SCHED_FUSED = 0, LBM_SCHED_UNFUSED = 1, LBM_SCHED_NO_GRAPH = 2 };
+ *  LBM_SCHED_SPLIT_E   (4) E separate: an Explosion kernel refreshes the
+ *                      level's explosion ghosts before its S / F kernel.
+ *  LBM_SCHED_SPLIT_A   (8) A separate, as a gather initiated from the coarse
+ *                      level after every fine Collision (raw sums into the
+ *                      coarse ghost slots; the paper's modified baseline).
+ *  LBM_SCHED_ATOMIC_A  (16) A fused into the fine Collision as a scatter
+ *                      atomic write (CA, Fig. 4c); the coarse
+ *                      kernel resets the ghost layer.  Summation order is not
+ *                      deterministic (results differ from the others by
+ *                      rounding only).
+ *  LBM_SCHED_SPLIT_O   (32) O's division by 2|B| as its own kernel before
+ *                      the coarse S / F (otherwise fused into the last
+ *                      Accumulate, or pre-scaled atomic terms).
+ * The paper's configurations: Fig. 4b modified baseline = UNFUSED | SPLIT_E |
+ * SPLIT_A | SPLIT_O; 4c = UNFUSED | SPLIT_E | ATOMIC_A | SPLIT_O; 4d (SE
+ * fused) = UNFUSED | SPLIT_A | SPLIT_O; 4e (CA, SE, SO fused) = UNFUSED |
+ * ATOMIC_A; 4f (CASE and SO fused) = ATOMIC_A.  All non-atomic schedules are
+ * bitwise identical to LBM_SCHED_FUSED.  Every bit except NO_GRAPH is single
+ * rank, paper variant only (LBM_E_UNSUPPORTED).  Switching at a coarse-step
+ * boundary is allowed (pending accumulations are rebuilt).  Takes effect at
+ * the next lbm_step; synchronises the grid's stream. */
+enum {
+  LBM_SCHED_FUSED = 0,
+  LBM_SCHED_UNFUSED = 1,
+  LBM_SCHED_NO_GRAPH = 2,
+  LBM_SCHED_SPLIT_E = 4,
+  LBM_SCHED_SPLIT_A = 8,
+  LBM_SCHED_ATOMIC_A = 16,
+  LBM_SCHED_SPLIT_O = 32
+};
 lbm_status lbm_set_schedule(lbm_grid* g, int32_t mode);
 
 /* Checkpoint / resume.  The state at a coarse-step

@@ -240,7 +240,7 @@ def cavity4_kbc(size: str = "full", collision: str = "kbc") -> Problem:
     )
 
 
-def tunnel4(scale: int = 1) -> Problem:
+def tunnel4(scale: int = 1, nu3: float = 0.004) -> Problem:
     """cfg5: D3Q19 BGK airplane-like virtual wind tunnel, coarse 200x105x105
     (1600x840x840 effective; reading R-A20), 4 levels.  Body in finest units:
     fuselage cylinder r=32, axis x in [400,880), centre (y,z)=(420,420); wing
@@ -248,7 +248,8 @@ def tunnel4(scale: int = 1) -> Problem:
     (coarse units): L1 x[22,138) y[20,85) z[0,105); L2 x[38,122) y[36,69)
     z[15,90); L3 x[46,114) y[44,61) z[23,82).  Inlet/outflow/walls as cfg3;
     nu_3 = 0.004 => nu_0 = nu_3/8.  scale=s divides every length by s (s in
-    {1, 5}: s=5 gives a 40x21x21 coarse grid for parity tests)."""
+    {1, 5}: s=5 gives a 40x21x21 coarse grid for parity tests); nu3 != 0.004
+    gives the same geometry at another viscosity (a lower-Re parity case)."""
     s = scale
 
     def d(v):
@@ -279,10 +280,10 @@ def tunnel4(scale: int = 1) -> Problem:
     wz = (zs >= 220.0 / s) & (zs < 620.0 / s)
     body |= wx[:, None, None] & wy[None, :, None] & wz[None, None, :]
     sub[body] = CLS_WALL
-    nu3 = 0.004
     nu0 = nu3 / 8.0
     return Problem(
-        name="tunnel4" + (f"_s{s}" if s != 1 else ""), nx=n[0], ny=n[1], nz=n[2], masks=masks,
+        name="tunnel4" + (f"_s{s}" if s != 1 else "") + (f"_nu{nu3:g}" if nu3 != 0.004 else ""),
+        nx=n[0], ny=n[1], nz=n[2], masks=masks,
         face_bc=(CLS_LID, CLS_OUT, CLS_WALL, CLS_WALL, CLS_WALL, CLS_WALL),
         Q=19, collision="bgk", omega0=1.0 / (3 * nu0 + 0.5),
         bc={CLS_WALL: (BC_NOSLIP, (0.0, 0.0, 0.0)), CLS_LID: (BC_VELOCITY, (0.05, 0.0, 0.0)),

@@ -63,6 +63,8 @@ struct DevLevel {
   uint32_t* ghost_fill = nullptr;
   uint32_t* coal_fill = nullptr;
   uint32_t* coal_cand = nullptr;
+  uint32_t* sc_qoff = nullptr;    // atomic Accumulate (ablation) scatter lists
+  uint32_t* sc_items = nullptr;
   uint32_t* vfill = nullptr;   // volumetric variant lists (grid_builder.h)
   uint32_t* vavg = nullptr;
   void* vtemp = nullptr;
@@ -97,6 +99,7 @@ struct lbm_grid {
   bool init_locked = false;  // a step ran since the last init_uniform
   bool broken = false;
   int sched = LBM_SCHED_FUSED;  // lbm_set_schedule
+  bool pdl = true;              // programmatic dependent launch of F_L^k after its gather (LBMR_NO_PDL=1: off)
   int64_t steps = 0;
   int64_t device_bytes = 0;
   std::vector<void*> allocs;
@@ -254,11 +257,85 @@ StepParams<T> make_params(const lbm_grid* g, int L, int64_t k) {
   return p;
 }
 
+// Schedule bits (lbmr.h LBM_SCHED_*), DESIGN.md §14:
+//   UNFUSED    C and S of a level-substep as two kernels (S_L^k, in-place C)
+//   SPLIT_E    Explosion as its own kernel E_L^k before S/F_L^k instead of the
+//              trailing CTAs of the level's previous kernel
+//   SPLIT_A    Accumulate as its own gather kernel after every fine Collision
+//              (raw sums into the coarse ghost slots, initiated from the coarse
+//              level: the paper's modified baseline)
+//   ATOMIC_A   Accumulate as a scatter atomic write fused into the fine
+//              Collision (CA fusion, Fig. 4c); the coarse kernel's
+//              trailing CTAs reset the accumulators it no longer needs
+//   SPLIT_O    Coalescence's division by 2|B| as its own kernel O_L^k before
+//              the coarse S/F (otherwise fused: into the last gather, or
+//              pre-scaled atomic terms)
+// The product schedule (0) gathers A + A + O in one small kernel right before
+// F_L^k from the two retained fine buffers (deterministic, no atomics).
+constexpr int kAblationBits = LBM_SCHED_SPLIT_E | LBM_SCHED_SPLIT_A | LBM_SCHED_ATOMIC_A | LBM_SCHED_SPLIT_O;
+
+bool level_has_coal(const lbm_grid* g, int L) {
+  return L >= 0 && L + 1 < g->levels && !g->host[L].coal_fill.empty();
+}
+
+void launch_gather(lbm_grid* g, int L, const void* fa, const void* fb, void* dst, int mode) {
+  const HostLevel& H = g->host[L];
+  launch_coalesce(g->Q, g->prec, fa, fb, dst, g->dev[L].coal_fill, g->dev[L].coal_cand, H.coal_n[0], H.coal_n[1], mode,
+                  g->stream);
+}
+
+// ablation fields of the level-L launch producing C_L^{k+1} (k = 0: prologue)
 template <typename T>
-void launch_F_typed(lbm_grid* g, int L, int64_t k, int kind) {
+void ablation_params(lbm_grid* g, int L, int64_t k, StepParams<T>& p) {
+  const int s = g->sched;
+  if (s & LBM_SCHED_SPLIT_E) p.nghost = 0;
+  if (s & LBM_SCHED_ATOMIC_A) {
+    if (level_has_coal(g, L)) {  // reset the accumulators of dst (read by F_L^{k+1})
+      p.zero_list = g->dev[L].coal_fill;
+      p.nzero = (int32_t)g->host[L].coal_fill.size();
+    }
+    if (L > 0 && level_has_coal(g, L - 1) && !g->host[L].sc_items.empty()) {
+      p.sc_qoff = g->dev[L].sc_qoff;
+      p.sc_items = reinterpret_cast<const uint4*>(g->dev[L].sc_items);
+      p.acc = static_cast<T*>(g->dev[L - 1].pop[((k + 2) / 2) & 1]);  // C_{L-1}^{ceil((k+1)/2)}'s buffer
+      p.sc_scaled = (s & LBM_SCHED_SPLIT_O) ? 0 : 1;
+    }
+  }
+}
+
+// Explosion ghosts of C_L^k's buffer from C_{L-1}^{ceil(k/2)} (the E kernel)
+template <typename T>
+void refresh_ghosts(lbm_grid* g, int L, int64_t k) {
+  StepParams<T> e = make_params<T>(g, L, k);
+  e.dst = static_cast<T*>(g->dev[L].pop[k & 1]);
+  e.gsrc = static_cast<const T*>(g->dev[L - 1].pop[((k + 1) / 2) & 1]);
+  launch_level_step(g->Q, g->coll, g->prec, 5, &e, g->stream);
+}
+
+// SPLIT_A: after C_L^j was produced (j >= 1), accumulate it into the coarse
+// ghost slots C_{L-1}^{ceil(j/2)} reads: the first fine substep sets the sum,
+// the second adds (and divides unless SPLIT_O).
+void accumulate_after(lbm_grid* g, int L, int64_t j) {
+  if (!(g->sched & LBM_SCHED_SPLIT_A) || L == 0 || !level_has_coal(g, L - 1)) return;
+  void* coarse = g->dev[L - 1].pop[((j + 1) / 2) & 1];
+  const void* fine = g->dev[L].pop[j & 1];
+  if (j & 1) launch_gather(g, L - 1, fine, nullptr, coarse, 0);
+  else launch_gather(g, L - 1, nullptr, fine, coarse, kCoalFromDst | ((g->sched & LBM_SCHED_SPLIT_O) ? 0 : kCoalDivide));
+}
+
+// mid / mid_stamp (optional): an event recorded, or a timestamp written,
+// after the pre-kernels (coalescence gather, volumetric averages, ablation
+// kernels) and before the level kernel itself (per-level profiling)
+template <typename T>
+void launch_F_typed(lbm_grid* g, int L, int64_t k, int kind, cudaEvent_t mid = nullptr,
+                    unsigned long long* mid_stamp = nullptr) {
   StepParams<T> p = make_params<T>(g, L, k);
-  if (kind == 1) {  // prologue collision
+  const int sched = g->sched;
+  if (kind == 1) {  // prologue collision C_L^1
+    ablation_params<T>(g, L, 0, p);
+    if (sched & LBM_SCHED_SPLIT_E) p.nghost = (int32_t)(g->host[L].ghost_fill.size() / 3);  // initial ghosts
     launch_level_step(g->Q, g->coll, g->prec, 1, &p, g->stream);
+    accumulate_after(g, L, 1);
     return;
   }
   const HostLevel& H = g->host[L];
@@ -268,29 +345,46 @@ void launch_F_typed(lbm_grid* g, int L, int64_t k, int kind) {
     launch_vavg(g->Q, g->prec, g->dev[L].vavg, (int32_t)(H.vavg.size() / 36), g->dev[L].pop[k & 1],
                 g->dev[L + 1].pop[1], g->dev[L + 1].pop[0], g->bc_dev, g->face_dev, g->dev[L].vtemp, g->stream);
   // coalescence ghosts of C_L^k from C_{L+1}^{2k-1} and C_{L+1}^{2k} (both ready now)
-  if (L + 1 < g->levels && !H.coal_fill.empty()) {
+  if (level_has_coal(g, L)) {
     if (g->n_ranks > 1) {
       // the gather reads L+1 halo cells: it follows the neighbour wait of F_L^k,
       // which launch_level_step issues first; issue an explicit wait here instead
       launch_halo_wait(p.flags, p.has_nb[0], p.has_nb[1], g->stream);
     }
-    launch_coalesce(g->Q, g->prec, g->dev[L + 1].pop[1], g->dev[L + 1].pop[0], g->dev[L].pop[k & 1],
-                    g->dev[L].coal_fill, g->dev[L].coal_cand, H.coal_n[0], H.coal_n[1], g->stream);
+    void* dst = g->dev[L].pop[k & 1];
+    if (!(sched & (LBM_SCHED_SPLIT_A | LBM_SCHED_ATOMIC_A))) {
+      launch_gather(g, L, g->dev[L + 1].pop[1], g->dev[L + 1].pop[0], dst,
+                    (sched & LBM_SCHED_SPLIT_O) ? 0 : kCoalDivide);
+      // the product schedule: F_L^k is the programmatic dependent of the
+      // gather (its CTAs that do not pull coalescence ghosts overlap it)
+      p.pdl = (g->n_ranks == 1 && !(sched & (LBM_SCHED_UNFUSED | kAblationBits)) && g->pdl) ? 1 : 0;
+    }
+    if (sched & LBM_SCHED_SPLIT_O) launch_gather(g, L, nullptr, nullptr, dst, kCoalFromDst | kCoalDivide);  // O
   }
-  if (g->sched & LBM_SCHED_UNFUSED) {  // S_L^k then C_L^{k+1} in place (fusion ablation)
-    launch_level_step(g->Q, g->coll, g->prec, 3, &p, g->stream);
+  // E_L^k: refresh the ghosts of C_L^k's buffer from C_{L-1}^{ceil(k/2)}
+  if ((sched & LBM_SCHED_SPLIT_E) && L > 0 && !H.ghost_fill.empty()) refresh_ghosts<T>(g, L, k);
+  ablation_params<T>(g, L, k, p);
+  if (mid) cudaEventRecord(mid, g->stream);
+  if (mid_stamp) launch_stamp(mid_stamp, 0, g->stream);
+  if (sched & LBM_SCHED_UNFUSED) {  // S_L^k then C_L^{k+1} in place (fusion ablation)
+    StepParams<T> sp = p;  // the stream half: no scatter (nothing collided yet)
+    sp.sc_qoff = nullptr;
+    launch_level_step(g->Q, g->coll, g->prec, 3, &sp, g->stream);
     StepParams<T> c = p;
     c.src = p.dst;
     c.nghost = 0;
+    c.nzero = 0;
     launch_level_step(g->Q, g->coll, g->prec, 4, &c, g->stream);
-    return;
+  } else {
+    launch_level_step(g->Q, g->coll, g->prec, 0, &p, g->stream);
   }
-  launch_level_step(g->Q, g->coll, g->prec, 0, &p, g->stream);
+  accumulate_after(g, L, k + 1);
 }
 
-void launch_F(lbm_grid* g, int L, int64_t k, int kind) {
-  if (g->prec == LBM_FP32) launch_F_typed<float>(g, L, k, kind);
-  else launch_F_typed<double>(g, L, k, kind);
+void launch_F(lbm_grid* g, int L, int64_t k, int kind, cudaEvent_t mid = nullptr,
+              unsigned long long* mid_stamp = nullptr) {
+  if (g->prec == LBM_FP32) launch_F_typed<float>(g, L, k, kind, mid, mid_stamp);
+  else launch_F_typed<double>(g, L, k, kind, mid, mid_stamp);
 }
 
 // The pipelined order of one coarse step n (0-based): list of (L, k).
@@ -515,6 +609,8 @@ static lbm_status build_host(const lbm_grid_desc* d, int32_t levels, const uint8
   in.Q = d->lattice;
   in.masks = masks;
   in.variant = d->variant;
+  in.align_blocks = getenv("LBMR_NO_BLOCK_ALIGN") ? 0 : 1;  // A/B switch for measurements
+  if (const char* o = getenv("LBMR_BLOCK_ORDER")) in.block_order = std::strcmp(o, "raster") == 0 ? 1 : 0;
   if (slab) {
     in.n0[0] = slab->desc.nx;
     in.periodic[0] = 0;
@@ -544,7 +640,8 @@ static int64_t planned_device_bytes(const std::vector<HostLevel>& host, int Q, s
     t += up(H.blkmap.size(), 4) + up(H.types.size(), 1) + up(H.origin.size(), 4) + up(H.nbr.size(), 4) +
          up(H.special_slot.size(), 4) + up(H.cellinfo.size(), 4) + up(H.bmask.size(), 4) + up(H.links.size(), 4) +
          up(H.coal.size(), 4) + up(H.bpeer.size(), 4) + up(H.ghost_fill.size(), 4) + up(H.coal_fill.size(), 4) +
-         up(H.coal_cand.size(), 4) + up(H.vfill.size(), 4) + up(H.vavg.size(), 4) + al((H.vavg.size() / 36) * ts) +
+         up(H.coal_cand.size(), 4) + up(H.sc_qoff.size(), 4) + up(H.sc_items.size(), 4) + up(H.vfill.size(), 4) +
+         up(H.vavg.size(), 4) + al((H.vavg.size() / 36) * ts) +
          2 * al((size_t)H.nfluid * Q * kCells * ts);
   if (n_ranks > 1) t += al(4 * sizeof(unsigned long long));
   t += al(sizeof(BCEntry) * 256) + al(32);
@@ -565,6 +662,7 @@ static void fill_info(const std::vector<HostLevel>& host, int Q, int prec, int n
     if (!host[L].coal_fill.empty()) info->launches_per_step += ((int64_t)1 << L) * (n_ranks > 1 ? 2 : 1);
     if (!host[L].vavg.empty()) info->launches_per_step += (int64_t)2 << L;
     info->leaves[L] = host[L].leaves;
+    for (int a = 0; a < 3; ++a) info->block_offset[L][a] = host[L].off[a];
     info->blocks[L] = host[L].nfluid;
     info->special_blocks[L] = host[L].nspecial;
     info->special_cells[L] = host[L].special_cells;
@@ -607,6 +705,7 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
   g->coll = d->collision;
   g->prec = d->precision;
   g->tsize = d->precision == LBM_FP32 ? 4 : 8;
+  g->pdl = getenv("LBMR_NO_PDL") == nullptr;
   for (int c = 0; c < 256; ++c) {
     g->bc_host[c].kind = LBM_BC_NOSLIP;
     g->bc_host[c].pad_ = 0;
@@ -681,6 +780,8 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     if ((s = dev_upload(g, &D.ghost_fill, H.ghost_fill))) return cleanup(s);
     if ((s = dev_upload(g, &D.coal_fill, H.coal_fill))) return cleanup(s);
     if ((s = dev_upload(g, &D.coal_cand, H.coal_cand))) return cleanup(s);
+    if ((s = dev_upload(g, &D.sc_qoff, H.sc_qoff))) return cleanup(s);
+    if ((s = dev_upload(g, &D.sc_items, H.sc_items))) return cleanup(s);
     if ((s = dev_upload(g, &D.vfill, H.vfill))) return cleanup(s);
     if ((s = dev_upload(g, &D.vavg, H.vavg))) return cleanup(s);
     if ((s = dev_alloc(g, &D.vtemp, (H.vavg.size() / 36) * g->tsize))) return cleanup(s);
@@ -766,8 +867,6 @@ static lbm_status init_level(lbm_grid* g, int L, const double* rho, const double
 #pragma omp parallel for schedule(static)
     for (int32_t i = 0; i < nb; ++i) {
       const int32_t b = b0 + i;
-      const int64_t ox = (int64_t)H.origin[3 * b] * kBlock, oy = (int64_t)H.origin[3 * b + 1] * kBlock,
-                    oz = (int64_t)H.origin[3 * b + 2] * kBlock;
       for (int l = 0; l < kCells; ++l) {
         const size_t k = (size_t)i * kCells + l;
         r[k] = rho0;
@@ -775,7 +874,7 @@ static lbm_status init_level(lbm_grid* g, int L, const double* rho, const double
         v[3 * k + 1] = u0 ? u0[1] : 0.0;
         v[3 * k + 2] = u0 ? u0[2] : 0.0;
         if (!(rho || u) || H.types[(size_t)b * kCells + l] != kFluid) continue;
-        const int64_t x = ox + (l & 7), y = oy + ((l >> 3) & 7), z = oz + (l >> 6);
+        const int64_t x = H.cell_x(b, l), y = H.cell_y(b, l), z = H.cell_z(b, l);
         if (x < H.owned_lo || x >= H.owned_hi) continue;  // halo cells come from the neighbour
         const int64_t c = ((x - H.owned_lo) * H.n[1] + y) * H.n[2] + z;
         if (rho) r[k] = rho[c];
@@ -862,9 +961,14 @@ lbm_status lbm_set_schedule(lbm_grid* g, int32_t mode) {
   g_err.clear();
   if (!g) return fail(LBM_E_INVAL, "NULL grid");
   DeviceGuard dg_(g);
-  if (mode < 0 || mode > (LBM_SCHED_UNFUSED | LBM_SCHED_NO_GRAPH)) return fail(LBM_E_INVAL, "bad schedule mode");
-  if ((mode & LBM_SCHED_UNFUSED) && g->n_ranks > 1)
-    return fail(LBM_E_UNSUPPORTED, "the unfused schedule is single-rank only");
+  const int all = LBM_SCHED_UNFUSED | LBM_SCHED_NO_GRAPH | kAblationBits;
+  if (mode < 0 || (mode & ~all)) return fail(LBM_E_INVAL, "bad schedule mode");
+  if ((mode & (LBM_SCHED_UNFUSED | kAblationBits)) && g->n_ranks > 1)
+    return fail(LBM_E_UNSUPPORTED, "the ablation schedules are single-rank only");
+  if ((mode & kAblationBits) && g->desc.variant != LBM_VARIANT_PAPER)
+    return fail(LBM_E_UNSUPPORTED, "the E/A/O ablation schedules need the paper variant");
+  if ((mode & LBM_SCHED_SPLIT_A) && (mode & LBM_SCHED_ATOMIC_A))
+    return fail(LBM_E_INVAL, "SPLIT_A and ATOMIC_A are two forms of the same Accumulate: choose one");
   if (mode == g->sched) return LBM_OK;
   CUDA_TRY(cudaStreamSynchronize(g->stream));
   for (int p = 0; p < 2; ++p)
@@ -872,7 +976,36 @@ lbm_status lbm_set_schedule(lbm_grid* g, int32_t mode) {
       cudaGraphExecDestroy(g->graph[p]);
       g->graph[p] = nullptr;
     }
+  const int acc_old = g->sched & (LBM_SCHED_SPLIT_A | LBM_SCHED_ATOMIC_A | LBM_SCHED_SPLIT_O);
+  const bool leave_split_e = (g->sched & LBM_SCHED_SPLIT_E) && !(mode & LBM_SCHED_SPLIT_E);
   g->sched = mode;
+  if (!g->needs_prologue && leave_split_e) {
+    // under SPLIT_E the explosion ghosts of the current buffers are refreshed
+    // by the E kernel right before they are read; the fused kernels expect the
+    // previous kernel to have done it: refresh them now
+    for (int L = 1; L < g->levels; ++L) {
+      if (g->host[L].ghost_fill.empty()) continue;
+      const int64_t k = (g->steps << L) + 1;  // next substep of level L
+      if (g->prec == LBM_FP32) refresh_ghosts<float>(g, L, k);
+      else refresh_ghosts<double>(g, L, k);
+    }
+    CUDA_TRY(cudaGetLastError());
+  }
+  const int acc_new = mode & (LBM_SCHED_SPLIT_A | LBM_SCHED_ATOMIC_A | LBM_SCHED_SPLIT_O);
+  if (!g->needs_prologue && acc_new != acc_old && (mode & (LBM_SCHED_SPLIT_A | LBM_SCHED_ATOMIC_A))) {
+    // At a coarse-step boundary the first fine substep of every coarse
+    // level's next substep has run already: its accumulation (kept implicitly
+    // in the fine buffer by the product schedule) is rebuilt in the form the
+    // new schedule expects in the coarse ghost slots.
+    for (int L = 0; L + 1 < g->levels; ++L) {
+      if (!level_has_coal(g, L)) continue;
+      const int64_t k = (g->steps << L) + 1;  // next substep of level L
+      const bool pre_scaled = (mode & LBM_SCHED_ATOMIC_A) && !(mode & LBM_SCHED_SPLIT_O);
+      launch_gather(g, L, g->dev[L + 1].pop[1], nullptr, g->dev[L].pop[k & 1], pre_scaled ? kCoalDivide : 0);
+    }
+    CUDA_TRY(cudaGetLastError());
+    CUDA_TRY(cudaStreamSynchronize(g->stream));
+  }
   return LBM_OK;
 }
 
@@ -979,50 +1112,111 @@ lbm_status lbm_checkpoint_load(lbm_grid* g, const void* host, int64_t size) {
   return LBM_OK;
 }
 
-lbm_status lbm_profile_levels(lbm_grid* g, int32_t n, double* ms_per_level, int64_t* launches_per_level) {
+lbm_status lbm_profile_step(lbm_grid* g, int32_t n, double* level_ms, double* gather_ms, int64_t* launches_per_level) {
   g_err.clear();
   if (!g) return fail(LBM_E_INVAL, "NULL grid");
   DeviceGuard dg_(g);
   if (g->broken) return fail(LBM_E_STATE, "grid is in an error state");
+  if (n < 0) return fail(LBM_E_INVAL, "n_coarse must be >= 0");
   for (int sd = 0; sd < 2; ++sd)
     if (g->n_ranks > 1 && g->has_nb[sd] && !g->connected[sd])
       return fail(LBM_E_STATE, "halo side " + std::to_string(sd) + " not connected");
   lbm_status s;
   if (g->needs_prologue && (s = run_prologue(g))) return s;
-  std::vector<std::pair<int, int64_t>> order;
-  std::vector<cudaEvent_t> ev;
-  std::vector<int> lev;
+  std::vector<double> lms(g->levels, 0.0), gms(g->levels, 0.0);
+  std::vector<int64_t> cnt(g->levels, 0);
+  // One instrumented graph per parity of the step index: the coarse step's
+  // launches in lbm_step's order, with a one-thread timestamp kernel node
+  // (device global timer) before each level kernel's pre-kernels
+  // (coalescence gather / volumetric averages / ablation kernels), between
+  // them and the level kernel, and after it.  Replayed like lbm_step's graph,
+  // so no host launch gaps are timed (CUDA event nodes in graphs cannot be
+  // timed).  Eager launches instead under LBM_SCHED_NO_GRAPH.
+  const size_t per = (size_t)1 << g->levels;  // > launches per coarse step
+  void *dv = nullptr, *hv = nullptr;
+  CUDA_TRY(cudaStreamSynchronize(g->stream));
+  if ((s = scratch_dev(g, 3 * per * sizeof(unsigned long long), &dv)) ||
+      (s = scratch_host(g, 3 * per * sizeof(unsigned long long), &hv)))
+    return s;
+  unsigned long long* ts = static_cast<unsigned long long*>(dv);
+  const unsigned long long* th = static_cast<const unsigned long long*>(hv);
+  std::vector<std::pair<int, int64_t>> order[2];
+  cudaGraphExec_t ge[2] = {nullptr, nullptr};
+  auto cleanup = [&]() {
+    for (int p = 0; p < 2; ++p)
+      if (ge[p]) cudaGraphExecDestroy(ge[p]);
+  };
+  auto issue = [&](int par) {
+    for (size_t j = 0; j < order[par].size(); ++j) {
+      launch_stamp(ts, (int)(3 * j), g->stream);
+      launch_F(g, order[par][j].first, order[par][j].second, 0, nullptr, ts + 3 * j + 1);
+      launch_stamp(ts, (int)(3 * j + 2), g->stream);
+    }
+  };
+  const bool eager = (g->sched & LBM_SCHED_NO_GRAPH) != 0;
   for (int i = 0; i < n; ++i) {
-    step_order(g->levels, g->steps, order);
-    for (auto& lk : order) {
-      cudaEvent_t a, b;
-      CUDA_TRY(cudaEventCreate(&a));
-      CUDA_TRY(cudaEventCreate(&b));
-      CUDA_TRY(cudaEventRecord(a, g->stream));
-      launch_F(g, lk.first, lk.second, 0);
-      CUDA_TRY(cudaEventRecord(b, g->stream));
-      ev.push_back(a);
-      ev.push_back(b);
-      lev.push_back(lk.first);
+    const int par = (int)(g->steps & 1);
+    step_order(g->levels, g->steps, order[par]);
+    if (eager) {
+      issue(par);
+    } else {
+      if (!ge[par]) {
+        if (cudaStreamBeginCapture(g->stream, cudaStreamCaptureModeThreadLocal) != cudaSuccess) {
+          cleanup();
+          return fail(LBM_E_CUDA, "profile capture");
+        }
+        issue(par);
+        cudaGraph_t graph = nullptr;
+        cudaError_t le = cudaGetLastError();
+        cudaError_t ce = cudaStreamEndCapture(g->stream, &graph);
+        if (le != cudaSuccess || ce != cudaSuccess) {
+          if (graph) cudaGraphDestroy(graph);
+          cleanup();
+          return fail(LBM_E_CUDA, std::string("profile capture: ") + cudaGetErrorString(le != cudaSuccess ? le : ce));
+        }
+        cudaError_t ie = cudaGraphInstantiate(&ge[par], graph, 0);
+        cudaGraphDestroy(graph);
+        if (ie != cudaSuccess) {
+          cleanup();
+          return fail(LBM_E_CUDA, std::string("profile instantiate: ") + cudaGetErrorString(ie));
+        }
+      }
+      if (cudaGraphLaunch(ge[par], g->stream) != cudaSuccess) {
+        cleanup();
+        return fail(LBM_E_CUDA, "profile graph launch");
+      }
+    }
+    cudaMemcpyAsync(hv, ts, 3 * order[par].size() * sizeof(unsigned long long), cudaMemcpyDeviceToHost, g->stream);
+    cudaError_t se = cudaStreamSynchronize(g->stream);
+    if (se != cudaSuccess) {
+      cleanup();
+      g->broken = true;
+      return fail(LBM_E_CUDA, std::string("profile step: ") + cudaGetErrorString(se));
+    }
+    for (size_t j = 0; j < order[par].size(); ++j) {
+      const int L = order[par][j].first;
+      gms[L] += (double)(th[3 * j + 1] - th[3 * j]) * 1e-6;
+      lms[L] += (double)(th[3 * j + 2] - th[3 * j + 1]) * 1e-6;
+      cnt[L] += 1;
     }
     ++g->steps;
   }
-  CUDA_TRY(cudaGetLastError());
-  CUDA_TRY(cudaStreamSynchronize(g->stream));
-  std::vector<double> ms(g->levels, 0.0);
-  std::vector<int64_t> cnt(g->levels, 0);
-  for (size_t i = 0; i < lev.size(); ++i) {
-    float t = 0;
-    CUDA_TRY(cudaEventElapsedTime(&t, ev[2 * i], ev[2 * i + 1]));
-    ms[lev[i]] += t;
-    cnt[lev[i]] += 1;
-  }
-  for (auto e : ev) cudaEventDestroy(e);
+  cleanup();
   for (int L = 0; L < g->levels; ++L) {
-    if (ms_per_level) ms_per_level[L] = ms[L];
+    if (level_ms) level_ms[L] = lms[L];
+    if (gather_ms) gather_ms[L] = gms[L];
     if (launches_per_level) launches_per_level[L] = cnt[L];
   }
   g->init_locked = true;
+  return LBM_OK;
+}
+
+lbm_status lbm_profile_levels(lbm_grid* g, int32_t n, double* ms_per_level, int64_t* launches_per_level) {
+  std::vector<double> lms(g ? g->levels : 1), gms(g ? g->levels : 1);
+  lbm_status s = lbm_profile_step(g, n, lms.data(), gms.data(), launches_per_level);
+  if (s) return s;
+  for (int L = 0; L < g->levels; ++L)
+    if (ms_per_level) ms_per_level[L] = lms[L] + gms[L];
   return LBM_OK;
 }
 
@@ -1067,11 +1261,9 @@ lbm_status lbm_macroscopic(lbm_grid* g, int32_t L, double* rho, double* u) {
 #pragma omp parallel for schedule(static)
     for (int32_t i = 0; i < nb; ++i) {
       const int32_t b = b0 + i;
-      const int64_t ox = (int64_t)H.origin[3 * b] * kBlock, oy = (int64_t)H.origin[3 * b + 1] * kBlock,
-                    oz = (int64_t)H.origin[3 * b + 2] * kBlock;
       for (int l = 0; l < kCells; ++l) {
         if (H.types[(size_t)b * kCells + l] != kFluid) continue;
-        const int64_t x = ox + (l & 7), y = oy + ((l >> 3) & 7), z = oz + (l >> 6);
+        const int64_t x = H.cell_x(b, l), y = H.cell_y(b, l), z = H.cell_z(b, l);
         if (x < H.owned_lo || x >= H.owned_hi) continue;
         const int64_t c = ((x - H.owned_lo) * H.n[1] + y) * H.n[2] + z;
         const size_t k = (size_t)i * kCells + l;
@@ -1100,9 +1292,9 @@ lbm_status lbm_probe(lbm_grid* g, int32_t L, int64_t n, const int64_t* xyz, doub
     if (x < 0 || x >= gnx || y < 0 || y >= H.n[1] || z < 0 || z >= H.n[2]) continue;
     x -= xoff;
     if (x < H.owned_lo || x >= H.owned_hi) continue;  // another rank's cell
-    const int32_t b = H.blkmap[((x >> 3) * H.nb[1] + (y >> 3)) * H.nb[2] + (z >> 3)];
+    const int32_t b = H.block_at(x, y, z);
     if (b < 0 || b >= H.nlaunch) continue;
-    const int l = (int)((x & 7) + 8 * (y & 7) + 64 * (z & 7));
+    const int l = H.local_at(x, y, z);
     if (H.types[(size_t)b * kCells + l] != kFluid) continue;
     cell[i] = (int64_t)b * kCells + l;
   }
@@ -1375,10 +1567,10 @@ lbm_status lbm_halo_plan(const lbm_grid_desc* d, int32_t levels, const uint8_t* 
     if (!xyz) return;
     for (size_t i = 0; i < v.size() && (int64_t)i < capacity; ++i) {
       const uint32_t b = v[i] >> 9, l = v[i] & 511u;
-      const int64_t x = (int64_t)H.origin[3 * b] * kBlock + (l & 7);
+      const int64_t x = H.cell_x((int32_t)b, (int)l);
       xyz[3 * i] = (((int64_t)slab.x_lo << level) + x + gn) % gn;
-      xyz[3 * i + 1] = (int64_t)H.origin[3 * b + 1] * kBlock + ((l >> 3) & 7);
-      xyz[3 * i + 2] = (int64_t)H.origin[3 * b + 2] * kBlock + (l >> 6);
+      xyz[3 * i + 1] = H.cell_y((int32_t)b, (int)l);
+      xyz[3 * i + 2] = H.cell_z((int32_t)b, (int)l);
     }
   };
   put(H.send[side], send_xyz);

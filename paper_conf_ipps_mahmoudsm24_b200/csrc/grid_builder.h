@@ -11,7 +11,12 @@ namespace lbmr {
 
 struct HostLevel {
   int64_t n[3] = {0, 0, 0};      // cells per axis
-  int32_t nb[3] = {0, 0, 0};     // blocks per axis (ceil(n/8))
+  int32_t nb[3] = {0, 0, 0};     // blocks per axis (ceil((n + off) / 8))
+  // block-grid offset per axis: level cell x lies in block (x + off) >> 3 at
+  // local position (x + off) & 7.  Chosen by the builder to put the level's
+  // fluid-region faces on block faces (whole 32-byte rows);
+  // always 0 on periodic axes.
+  int32_t off[3] = {0, 0, 0};
   int32_t nblocks = 0;           // stored blocks (fluid first)
   int32_t nfluid = 0;            // blocks holding >= 1 fluid leaf
   int32_t nspecial = 0;          // fluid blocks with a non-trivial cell
@@ -42,6 +47,11 @@ struct HostLevel {
   std::vector<uint32_t> coal_cand;    // SoA fine candidate population indices (level L+1), ~0u = empty:
                                       // [kCoalSlots][coal_n[0]] then [kCoalSlotsMax][coal_n[1]]
   int64_t coal_n[2] = {0, 0};         // entries with |B| <= kCoalSlots, and the others
+  // atomic form of Accumulate (ablation schedule LBM_SCHED_ATOMIC_A): this
+  // level's contributions to the coarser level's coalescence entries,
+  // grouped by the 128-cell quarter block of the contributing fine cell
+  std::vector<uint32_t> sc_qoff;      // [4 nfluid + 1] CSR offsets into sc_items
+  std::vector<uint32_t> sc_items;     // [n][4] {fine population index, coarse slot, |B|, 0}
   // volumetric variant: expressions are uint4 {pop index,
   // tag | nwall << 4 | wall0 << 8, wall1 | wall2 << 16, 0} (lattice.h kVt*)
   std::vector<uint32_t> vfill;        // [n][8]: {dst pop index, 0, 0, 0, expr}: the second-substep ghost packets
@@ -49,6 +59,17 @@ struct HostLevel {
   std::vector<uint32_t> avg_base;     // host only: [nblocks*512] first vavg entry of an averaged cell, or ~0u
   std::vector<int32_t> plain_ids;     // fluid blocks without special cells (Morton order)
   std::vector<int32_t> special_ids;   // the others (Morton order)
+
+  // coordinate maps (cells in [0, n) per axis)
+  int32_t block_at(int64_t x, int64_t y, int64_t z) const {
+    return blkmap[(((x + off[0]) >> 3) * nb[1] + ((y + off[1]) >> 3)) * nb[2] + ((z + off[2]) >> 3)];
+  }
+  int local_at(int64_t x, int64_t y, int64_t z) const {
+    return (int)(((x + off[0]) & 7) + 8 * ((y + off[1]) & 7) + 64 * ((z + off[2]) & 7));
+  }
+  int64_t cell_x(int32_t b, int l) const { return (int64_t)origin[3 * b] * 8 + (l & 7) - off[0]; }
+  int64_t cell_y(int32_t b, int l) const { return (int64_t)origin[3 * b + 1] * 8 + ((l >> 3) & 7) - off[1]; }
+  int64_t cell_z(int32_t b, int l) const { return (int64_t)origin[3 * b + 2] * 8 + (l >> 6) - off[2]; }
 };
 
 struct BuildInput {
@@ -64,6 +85,8 @@ struct BuildInput {
   int32_t owned_lo0 = 0, owned_hi0 = -1;
   int32_t has_nb[2] = {0, 0};
   int32_t variant = 0;                // 0 paper's method, 1 volumetric ghost advection
+  int32_t align_blocks = 1;           // choose HostLevel::off (0: block grids start at cell 0)
+  int32_t block_order = 0;            // 0 Morton, 1 raster (grid_builder.cpp block_key)
 };
 
 // Returns 0 on success; otherwise an lbm_status code with `err` filled.

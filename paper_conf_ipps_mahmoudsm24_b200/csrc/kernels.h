@@ -60,6 +60,22 @@ struct StepParams {
   const uint32_t* vfill;
   int32_t nvfill;
   const T* vtemp;               // coarse averages of this level (kLinkTemp records)
+  // ---- fusion-ablation schedules (lbm_set_schedule) --------
+  // LBM_SCHED_ATOMIC_A (the paper's CA fusion): after colliding,
+  // this level's CTAs add their post-collision values into the coarse
+  // accumulators (the coalescence-ghost slots of C_{L-1}'s buffer `acc`) with
+  // atomics, and the trailing CTAs reset this level's own accumulators in dst
+  const uint32_t* zero_list;    // coalescence-ghost slots of dst to reset (nzero)
+  int32_t nzero;
+  const uint32_t* sc_qoff;      // [4 nfluid + 1] scatter items per 128-cell quarter block (CSR)
+  const uint4* sc_items;        // {fine population index, coarse slot, |B|, 0}
+  T* acc;                       // coarse buffer receiving the scatter (C_{L-1}^{ceil((k+1)/2)})
+  int32_t sc_scaled;            // 1: add v / (2|B|) (division fused), 0: add v (separate O kernel)
+  // 1: launched as the programmatic dependent (PDL) of the coalescence gather
+  // that fills this kernel's coalescence ghosts: CTAs of blocks that pull
+  // them (record word kRecCoalPull) wait for the gather at their start, all
+  // others at their end, so the gather overlaps the level kernel
+  int32_t pdl;
   // ---- x-slab partition (multi-GPU); unused when nbctas == 0 -------------
   int32_t nbctas;               // CTAs taking part in the halo protocol (cut-plane blocks, >= 1)
   int32_t nboundary;            // cut-plane blocks (stored and launched first)
@@ -76,8 +92,14 @@ struct StepParams {
 // / (2|B|) over the filled candidate slots of entry i (grid_builder.h
 // coal_cand: n_main entries with kCoalSlots slots, then n_ovf entries with
 // kCoalSlotsMax slots, structure-of-arrays).
+// mode (kCoal*): kCoalFromDst starts each sum from dst[fill[i]] instead of 0,
+// kCoalDivide divides the sum by 2|B|; fa / fb may be NULL (that source is
+// skipped).  The product schedule's gather is (fa, fb, kCoalDivide); the
+// ablation schedules split it into Accumulate (fa or fb only, no division)
+// and Coalescence O (no source, kCoalFromDst | kCoalDivide) kernels.
+enum { kCoalFromDst = 1, kCoalDivide = 2 };
 void launch_coalesce(int Q, int precision, const void* fa, const void* fb, void* dst, const uint32_t* fill,
-                     const uint32_t* cand, int64_t n_main, int64_t n_ovf, cudaStream_t s);
+                     const uint32_t* cand, int64_t n_main, int64_t n_ovf, int mode, cudaStream_t s);
 
 // rho / u (double) of n cells given by population cell index block*512+local
 // (-1 -> NaN), read from the post-collision buffer `pop`.
@@ -102,12 +124,16 @@ struct FaceTable {
 };
 void launch_bc_update(BCEntry* bc, int cls, BCEntry e, uint8_t* face_cls, FaceTable ft, cudaStream_t s);
 
+// One-thread kernel writing the device global timer (ns) into out[idx].
+void launch_stamp(unsigned long long* out, int idx, cudaStream_t s);
+
 // Force-load every kernel (see level_step.cu).
 void preload_kernels();
 
 // kind: 0 = fused stream+collide F_L^k, 1 = collide only (prologue C_L^1,
 // src -> dst), 3 = stream only S_L^k (unfused schedule, with the explosion
-// ghost refresh), 4 = collide dst in place (unfused schedule)
+// ghost refresh), 4 = collide dst in place (unfused schedule), 5 = Explosion
+// only: refresh the explosion ghosts of dst from gsrc (ablation E kernel)
 void launch_level_step(int Q, int collision, int precision, int kind, const void* params, cudaStream_t s);
 
 // g = f^eq(rho,u) - w on the fluid cells of `nfluid` blocks; rho/u compact

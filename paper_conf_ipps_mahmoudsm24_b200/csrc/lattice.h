@@ -43,11 +43,14 @@ constexpr unsigned kFluidBit = 1u << 31;
 // per-fluid-block record of 64 int32 (two 128-byte lines, one warp load
 // each): [0..26] neighbour block ids by nbr_slot (-1: none, outside, or a
 // block without fluid leaves), [27] special slot (-1 plain), [28..30] block
-// coordinates, [31] unused, [32+w] fluid-leaf mask of warp w (cells 32w..32w+31),
+// coordinates, [31] 1 if a fluid leaf of the block pulls a coalescence ghost
+// (waits for the gather kernel under programmatic dependent launch),
+// [32+w] fluid-leaf mask of warp w (cells 32w..32w+31),
 // [48+w] mask of the fluid leaves of warp w that have a slow link
 constexpr int kRec = 64;
 constexpr int kRecSlot = 27;
 constexpr int kRecOrigin = 28;
+constexpr int kRecCoalPull = 31;
 constexpr int kRecFluid = 32;
 constexpr int kRecSpecial = 48;
 // per special block: 16 words, word w = union over the fluid leaves of warp w

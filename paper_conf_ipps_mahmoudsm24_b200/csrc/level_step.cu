@@ -613,9 +613,40 @@ __device__ __forceinline__ void trail_fill(const StepParams<T>& P, int i) {
     const uint32_t* e = P.vfill + 8 * (size_t)i;
     P.dst[e[0]] = vexpr<Q, T>(e + 4, P.src, P.gsrc, nullptr, P.bc, P.face_cls);
   }
+  // ablation schedule LBM_SCHED_ATOMIC_A: reset the accumulators (coalescence
+  // ghost slots) the next fine collisions add into ("it will reset the
+  // ghost layer")
+  if (i < P.nzero) P.dst[__ldg(P.zero_list + i)] = T(0);
 }
 
 __host__ __device__ inline int trail_items(int nghost, int nvfill) { return nghost > nvfill ? nghost : nvfill; }
+template <typename T>
+__host__ __device__ inline int trail_count(const StepParams<T>& p) {
+  const int a = trail_items(p.nghost, p.nvfill);
+  return a > p.nzero ? a : p.nzero;
+}
+
+// Ablation schedule LBM_SCHED_ATOMIC_A (Fig. 4c, the paper's Accumulate as a
+// scatter atomic write fused into the Collision): the CTA that
+// just stored the post-collision values of cells [base, base + NT) of block
+// blk adds each value a coarse coalescence link needs into that link's
+// accumulator (the coarse ghost slot), v / (2|B|) when the division is fused
+// (no O kernel) or v.  Items are grouped per 128-cell quarter block, so a CTA
+// reads only values its own threads wrote (visible after the barrier).  At
+// most 8 fine cells add into one accumulator, so contention is low.
+template <typename T, int NT>
+__device__ __forceinline__ void accumulate_scatter(const StepParams<T>& P, int blk, int base) {
+  const unsigned q0 = (unsigned)blk * 4u + (unsigned)(base >> 7);
+  const unsigned a = __ldg(P.sc_qoff + q0), b = __ldg(P.sc_qoff + q0 + NT / 128);
+  if (a == b) return;  // CTA-uniform
+  __syncthreads();
+  for (unsigned i = a + threadIdx.x; i < b; i += NT) {
+    const uint4 it = __ldg(P.sc_items + i);
+    T v = P.dst[it.x];
+    if (P.sc_scaled) v = v / T(2 * it.z);
+    atomicAdd(P.acc + it.y, v);
+  }
+}
 
 // Minimum resident CTAs per SM (register budget 65536 / (256 * MINB)),
 // chosen per variant from ptxas -v and measurement.
@@ -818,6 +849,12 @@ struct StepCta {
   static constexpr int min_blocks = (PlainOcc<Q, T, COLL>::value * 256) / threads;
 };
 
+// Programmatic dependent launch (sm_90+): wait until the preceding kernel of
+// the stream (the coalescence gather) has completed and its writes are
+// visible; let the following kernel launch early.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_launch_dependents() { asm volatile("griddepcontrol.launch_dependents;" :::); }
+
 template <int Q, int COLL, typename T>
 __global__ void __launch_bounds__(StepCta<Q, COLL, T>::threads, StepCta<Q, COLL, T>::min_blocks)
     level_step_all(const StepParams<T> P) {
@@ -825,10 +862,17 @@ __global__ void __launch_bounds__(StepCta<Q, COLL, T>::threads, StepCta<Q, COLL,
   const int main = P.nfluid * PB;
   if ((int)blockIdx.x >= main) {  // trailing CTAs refresh the explosion ghosts
     trail_fill<Q, T>(P, ((int)blockIdx.x - main) * NT + threadIdx.x);
+    if (P.pdl) pdl_wait();  // this kernel completes only after the gather
     return;
   }
   const int b = (int)blockIdx.x;
+  // under PDL the gather may still be running: CTAs whose block pulls a
+  // coalescence ghost wait for it first, the others after their work
+  const bool early = P.pdl && __ldg(P.nbr + (b / PB) * kRec + kRecCoalPull) != 0;
+  if (early) pdl_wait();
   step_cell<Q, COLL, T, false, true, NT>(P, b / PB, (b % PB) * NT + threadIdx.x);
+  if (P.sc_qoff) accumulate_scatter<T, NT>(P, b / PB, (b % PB) * NT);
+  if (P.pdl && !early) pdl_wait();
 }
 
 // Partitioned variant: grid = 4 * max(nfluid, 1) quarter-block CTAs; the first nbctas run
@@ -884,7 +928,7 @@ __global__ void __launch_bounds__(kHaloCtaThreads, (PlainOcc<Q, T, COLL>::value 
     if (STREAM) step_cell<Q, COLL, T, true, true, NT>(P, blk, t);
     else collide_cell<Q, COLL, T, true>(P, blk, t);
   }
-  if (proto) halo_signal<T>(P, P.nbctas + halo_fill_ctas(trail_items(P.nghost, P.nvfill)));
+  if (proto) halo_signal<T>(P, P.nbctas + halo_fill_ctas(trail_count(P)));
 }
 
 template <int Q, int COLL, typename T>
@@ -894,6 +938,7 @@ __global__ void __launch_bounds__(256) level_collide(const StepParams<T> P) {
     return;
   }
   collide_cell<Q, COLL, T, false>(P, blockIdx.x >> 1, ((blockIdx.x & 1) << 8) | threadIdx.x);
+  if (P.sc_qoff) accumulate_scatter<T, 256>(P, blockIdx.x >> 1, (blockIdx.x & 1) << 8);
 }
 
 // Unfused schedule (fusion ablation, Fig.4 / Fig.9): S_L^k pulls
@@ -914,6 +959,15 @@ __global__ void __launch_bounds__(256, PlainOcc<Q, T, LBM_BGK>::value) level_str
 template <int Q, int COLL, typename T>
 __global__ void __launch_bounds__(256) level_collide_inplace(const StepParams<T> P) {
   collide_cell<Q, COLL, T, false, true>(P, blockIdx.x >> 1, ((blockIdx.x & 1) << 8) | threadIdx.x);
+  if (P.sc_qoff) accumulate_scatter<T, 256>(P, blockIdx.x >> 1, (blockIdx.x & 1) << 8);
+}
+
+// Ablation schedule LBM_SCHED_SPLIT_E: Explosion (Eq.10) as its own kernel,
+// refreshing the explosion ghosts of dst from the parent level's
+// post-collision state gsrc right before the level's streaming kernel.
+template <int Q, typename T>
+__global__ void __launch_bounds__(256) explosion_refresh(const StepParams<T> P) {
+  ghost_fill_one<Q, T>(P, (int)blockIdx.x * 256 + threadIdx.x);
 }
 
 // ---------------------------------------------------------------- init / macroscopic
@@ -1026,33 +1080,44 @@ void launch_probe(int Q, int precision, const void* pop, const int64_t* cell, in
 // plane; candidate slots structure-of-arrays (grid_builder.h coal_cand).
 // Fine candidates summed in candidate order, first substep then second, like
 // the oracle (Eq.11, n = 2|B|, R-A2/R-A3).
+// mode: kCoalFromDst / kCoalDivide (kernels.h); fa / fb may be NULL.  The
+// terms are added in the oracle's order (fa candidates, then fb candidates),
+// so the split Accumulate kernels of the ablation schedules reproduce the
+// one-kernel gather bitwise.
 template <typename T, int K>
-__device__ __forceinline__ void coalesce_one(const T* __restrict__ fa, const T* __restrict__ fb, T* __restrict__ dst,
-                                             uint32_t d, const uint32_t* __restrict__ cand, int64_t stride) {
+__device__ __forceinline__ void coalesce_one(const T* __restrict__ fa, const T* __restrict__ fb, T* dst, uint32_t d,
+                                             const uint32_t* __restrict__ cand, int64_t stride, int mode) {
   uint32_t c[K];
 #pragma unroll
   for (int m = 0; m < K; ++m) c[m] = __ldg(cand + m * stride);
-  T acc = T(0);
+  T acc = (mode & kCoalFromDst) ? dst[d] : T(0);
   unsigned cnt = 0;
 #pragma unroll
   for (int m = 0; m < K; ++m)
-    if (c[m] != ~0u) { acc += __ldg(fa + c[m]); ++cnt; }
+    if (c[m] != ~0u) {
+      if (fa) acc += __ldg(fa + c[m]);
+      ++cnt;
+    }
+  if (fb) {
 #pragma unroll
-  for (int m = 0; m < K; ++m)
-    if (c[m] != ~0u) acc += __ldg(fb + c[m]);
-  dst[d] = acc / T(2 * cnt);
+    for (int m = 0; m < K; ++m)
+      if (c[m] != ~0u) acc += __ldg(fb + c[m]);
+  }
+  dst[d] = (mode & kCoalDivide) ? acc / T(2 * cnt) : acc;
 }
 
 template <typename T>
-__global__ void __launch_bounds__(256) coalesce_kernel(const T* __restrict__ fa, const T* __restrict__ fb,
-                                                       T* __restrict__ dst, const uint32_t* __restrict__ fill,
-                                                       const uint32_t* __restrict__ cand, int64_t nmain, int64_t novf) {
+__global__ void __launch_bounds__(256) coalesce_kernel(const T* __restrict__ fa, const T* __restrict__ fb, T* dst,
+                                                       const uint32_t* __restrict__ fill,
+                                                       const uint32_t* __restrict__ cand, int64_t nmain, int64_t novf,
+                                                       int mode) {
+  pdl_launch_dependents();  // the level kernel after it may start (it waits where it needs us)
   const int64_t i = (int64_t)blockIdx.x * 256 + threadIdx.x;
   if (i < nmain) {
-    coalesce_one<T, kCoalSlots>(fa, fb, dst, __ldg(fill + i), cand + i, nmain);
+    coalesce_one<T, kCoalSlots>(fa, fb, dst, __ldg(fill + i), cand + i, nmain, mode);
   } else if (i < nmain + novf) {
     const int64_t j = i - nmain;
-    coalesce_one<T, kCoalSlotsMax>(fa, fb, dst, __ldg(fill + i), cand + kCoalSlots * nmain + j, novf);
+    coalesce_one<T, kCoalSlotsMax>(fa, fb, dst, __ldg(fill + i), cand + kCoalSlots * nmain + j, novf, mode);
   }
 }
 
@@ -1105,22 +1170,29 @@ void launch_bc_update(BCEntry* bc, int cls, BCEntry e, uint8_t* face_cls, FaceTa
   bc_update_kernel<<<1, 32, 0, s>>>(bc, cls, e, face_cls, ft);
 }
 
+// Profiling stamp (lbm_profile_step): one thread writes the device global
+// timer (ns) into out[idx]; as a graph kernel node between two level kernels
+// it runs after the first has completed and before the second starts.
+__global__ void stamp_kernel(unsigned long long* out, int idx) { out[idx] = globaltimer_ns(); }
+
+void launch_stamp(unsigned long long* out, int idx, cudaStream_t s) { stamp_kernel<<<1, 1, 0, s>>>(out, idx); }
+
 void launch_halo_wait(const unsigned long long* flags, int nb0, int nb1, cudaStream_t s) {
   halo_wait_kernel<<<1, 1, 0, s>>>(flags, nb0, nb1);
 }
 
 void launch_coalesce(int Q, int precision, const void* fa, const void* fb, void* dst, const uint32_t* fill,
-                     const uint32_t* cand, int64_t n_main, int64_t n_ovf, cudaStream_t s) {
+                     const uint32_t* cand, int64_t n_main, int64_t n_ovf, int mode, cudaStream_t s) {
   (void)Q;
   const int64_t n = n_main + n_ovf;
   if (n <= 0) return;
   const unsigned grid = (unsigned)((n + 255) / 256);
   if (precision == LBM_FP32)
     coalesce_kernel<float><<<grid, 256, 0, s>>>((const float*)fa, (const float*)fb, (float*)dst, fill, cand, n_main,
-                                                 n_ovf);
+                                                 n_ovf, mode);
   else
     coalesce_kernel<double><<<grid, 256, 0, s>>>((const double*)fa, (const double*)fb, (double*)dst, fill, cand,
-                                                  n_main, n_ovf);
+                                                  n_main, n_ovf, mode);
 }
 
 // ---------------------------------------------------------------- dispatch
@@ -1134,16 +1206,20 @@ static void launch_typed(int kind, const void* params, cudaStream_t s) {
   const StepParams<T>& p = *static_cast<const StepParams<T>*>(params);
   dim3 block(256);
   const size_t sm = slow_smem<Q, T>();
-  const int gc = ghost_ctas(trail_items(p.nghost, p.nvfill));
+  const int gc = ghost_ctas(trail_count(p));
+  if (kind == 5) {  // Explosion only (ablation E kernel)
+    if (p.nghost > 0) explosion_refresh<Q, T><<<dim3(ghost_ctas(p.nghost)), block, 0, s>>>(p);
+    return;
+  }
   if (p.nbctas > 0) {  // partitioned: always launched (the protocol must run)
     halo_wait_kernel<<<1, 1, 0, s>>>(p.flags, p.has_nb[0], p.has_nb[1]);
-    dim3 grid(kHaloCtasPerBlock * std::max(p.nfluid, 1) + halo_fill_ctas(trail_items(p.nghost, p.nvfill)));
+    dim3 grid(kHaloCtasPerBlock * std::max(p.nfluid, 1) + halo_fill_ctas(trail_count(p)));
     const size_t hs = (size_t)Q * kHaloCtaThreads * sizeof(T);
     if (kind == 1) level_step_halo<Q, COLL, T, false><<<grid, dim3(kHaloCtaThreads), 0, s>>>(p);
     else level_step_halo<Q, COLL, T, true><<<grid, dim3(kHaloCtaThreads), hs, s>>>(p);
     return;
   }
-  if (p.nfluid <= 0 && p.nghost <= 0 && p.nvfill <= 0) return;
+  if (p.nfluid <= 0 && trail_count(p) <= 0) return;
   if (kind == 1) {
     level_collide<Q, COLL, T><<<dim3(2 * p.nfluid + gc), block, 0, s>>>(p);
   } else if (kind == 3) {
@@ -1152,9 +1228,24 @@ static void launch_typed(int kind, const void* params, cudaStream_t s) {
     if (p.nfluid > 0) level_collide_inplace<Q, COLL, T><<<dim3(2 * p.nfluid), block, 0, s>>>(p);
   } else {
     constexpr int NT = StepCta<Q, COLL, T>::threads;
-    const int gct = (trail_items(p.nghost, p.nvfill) + NT - 1) / NT;
-    level_step_all<Q, COLL, T><<<dim3(p.nfluid * StepCta<Q, COLL, T>::per_block + gct), dim3(NT),
-                                 (size_t)Q * NT * sizeof(T), s>>>(p);
+    const int gct = (trail_count(p) + NT - 1) / NT;
+    const dim3 grid(p.nfluid * StepCta<Q, COLL, T>::per_block + gct), blk(NT);
+    const size_t smem = (size_t)Q * NT * sizeof(T);
+    if (p.pdl) {
+      cudaLaunchConfig_t cfg = {};
+      cfg.gridDim = grid;
+      cfg.blockDim = blk;
+      cfg.dynamicSmemBytes = smem;
+      cfg.stream = s;
+      cudaLaunchAttribute attr[1];
+      attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+      attr[0].val.programmaticStreamSerializationAllowed = 1;
+      cfg.attrs = attr;
+      cfg.numAttrs = 1;
+      cudaLaunchKernelEx(&cfg, level_step_all<Q, COLL, T>, p);
+    } else {
+      level_step_all<Q, COLL, T><<<grid, blk, smem, s>>>(p);
+    }
   }
 }
 
@@ -1176,6 +1267,7 @@ static void preload_variant() {
   cudaFuncGetAttributes(&a, level_collide<Q, COLL, T>);
   cudaFuncGetAttributes(&a, level_step_halo<Q, COLL, T, true>);
   cudaFuncGetAttributes(&a, level_step_halo<Q, COLL, T, false>);
+  cudaFuncGetAttributes(&a, explosion_refresh<Q, T>);
 }
 
 void preload_kernels() {
@@ -1187,6 +1279,7 @@ void preload_kernels() {
   preload_variant<27, LBM_KBC, double>();
   cudaFuncAttributes a;
   cudaFuncGetAttributes(&a, halo_wait_kernel);
+  cudaFuncGetAttributes(&a, stamp_kernel);
   cudaFuncGetAttributes(&a, bc_update_kernel);
   cudaFuncGetAttributes(&a, coalesce_kernel<float>);
   cudaFuncGetAttributes(&a, probe_kernel<19, float>);

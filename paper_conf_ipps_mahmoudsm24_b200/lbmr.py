@@ -23,6 +23,16 @@ BGK, KBC = 0, 1
 FP32, FP64 = 0, 1
 BC_NOSLIP, BC_VELOCITY, BC_OUTFLOW = 0, 1, 2
 SCHED_FUSED, SCHED_UNFUSED, SCHED_NO_GRAPH = 0, 1, 2
+SCHED_SPLIT_E, SCHED_SPLIT_A, SCHED_ATOMIC_A, SCHED_SPLIT_O = 4, 8, 16, 32
+# the paper's Fig. 4 configurations as schedule bit sets
+FIG4 = {
+    "4b": SCHED_UNFUSED | SCHED_SPLIT_E | SCHED_SPLIT_A | SCHED_SPLIT_O,  # modified baseline: C, A, S, E, O
+    "4c": SCHED_UNFUSED | SCHED_SPLIT_E | SCHED_ATOMIC_A | SCHED_SPLIT_O,  # CA fused (atomic Accumulate)
+    "4d": SCHED_UNFUSED | SCHED_SPLIT_A | SCHED_SPLIT_O,  # SE fused
+    "4e": SCHED_UNFUSED | SCHED_ATOMIC_A,  # CA, SE and SO fused
+    "4f": SCHED_ATOMIC_A,  # CASE and SO fused (the paper's design)
+    "product": SCHED_FUSED,  # fused level kernels, gather A+A+O (deterministic)
+}
 VARIANT_PAPER, VARIANT_VOLUMETRIC = 0, 1
 
 
@@ -54,6 +64,7 @@ class GridInfo(ctypes.Structure):
         ("total_blocks", ctypes.c_int64 * 16),
         ("device_bytes", ctypes.c_int64), ("steps_done", ctypes.c_int64),
         ("launches_per_step", ctypes.c_int64),
+        ("block_offset", (ctypes.c_int32 * 3) * 16),
     ]
 
 
@@ -62,7 +73,7 @@ EXPORTS = ["lbm_grid_create", "lbm_set_bc", "lbm_init_equilibrium", "lbm_init_un
            "lbm_grid_destroy", "lbm_last_error", "lbm_version", "lbm_grid_analyze", "lbm_schedule",
            "lbm_lattice_table", "lbm_omega_level", "lbm_partition_cuts", "lbm_grid_slab", "lbm_halo_export",
            "lbm_halo_connect", "lbm_halo_connect_local", "lbm_halo_plan", "lbm_set_schedule",
-           "lbm_checkpoint_size", "lbm_checkpoint_save", "lbm_checkpoint_load", "lbm_probe", "lbm_debug_flags"]
+           "lbm_checkpoint_size", "lbm_checkpoint_save", "lbm_checkpoint_load", "lbm_probe", "lbm_debug_flags", "lbm_profile_step"]
 
 _lib = None
 
@@ -88,6 +99,7 @@ def load_library(path: str = LIB_PATH):
     lib.lbm_stats.argtypes = [P, lp, dp]
     lib.lbm_grid_get_info.argtypes = [P, ctypes.POINTER(GridInfo)]
     lib.lbm_profile_levels.argtypes = [P, ctypes.c_int32, dp, lp]
+    lib.lbm_profile_step.argtypes = [P, ctypes.c_int32, dp, dp, lp]
     lib.lbm_synchronize.argtypes = [P]
     lib.lbm_grid_destroy.argtypes = [P]
     lib.lbm_grid_destroy.restype = None
@@ -353,7 +365,8 @@ class Grid:
         return gi
 
     def set_schedule(self, mode: int):
-        """SCHED_FUSED (default) | SCHED_UNFUSED | SCHED_NO_GRAPH (bit flags)."""
+        """Bit flags SCHED_* (lbmr.h lbm_set_schedule); FIG4 names the paper's
+        Fig. 4 configurations."""
         _check(self.lib.lbm_set_schedule(self.h, int(mode)))
 
     def checkpoint_size(self) -> int:
@@ -376,6 +389,16 @@ class Grid:
         out = (ctypes.c_ulonglong * 4)()
         _check(self.lib.lbm_debug_flags(self.h, out))
         return [int(v) for v in out]
+
+    def profile_step(self, n_coarse: int):
+        """(level_ms[L], gather_ms[L], launches[L]) summed over n_coarse
+        instrumented coarse steps (lbm_profile_step)."""
+        lms = np.zeros(self.levels)
+        gms = np.zeros(self.levels)
+        cnt = np.zeros(self.levels, dtype=np.int64)
+        _check(self.lib.lbm_profile_step(self.h, int(n_coarse), _dp(lms), _dp(gms),
+                                         cnt.ctypes.data_as(ctypes.POINTER(ctypes.c_int64))))
+        return lms, gms, cnt
 
     def profile_levels(self, n_coarse: int):
         ms = np.zeros(self.levels)

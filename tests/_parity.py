@@ -1,9 +1,31 @@
 """Helpers for GPU-vs-oracle parity (SURVEY §8(c.5) error definitions)."""
 from __future__ import annotations
 
+import json
+import os
+import time
+
 import numpy as np
 
 import oracle
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+# every GPU parity check appends its measured errors here (gpurun merges
+# gpurun_out/ back; tools/parity_table.py turns it into
+# profiles/r02_parity_errors.json)
+PARITY_LOG = os.environ.get("LBMR_PARITY_LOG", os.path.join(ROOT, "gpurun_out", "parity_errors.jsonl"))
+
+
+def record(test: str, config: str, steps: int, precision: int, err_rho: float, err_u: float, **extra):
+    """Append one measured (err_rho, err_u) to the parity log (best effort)."""
+    try:
+        os.makedirs(os.path.dirname(PARITY_LOG), exist_ok=True)
+        line = {"test": test, "config": config, "steps": int(steps), "precision": "fp64" if precision else "fp32",
+                "err_rho": float(err_rho), "err_u": float(err_u), "bar": TOL[precision], "time": time.time(), **extra}
+        with open(PARITY_LOG, "a") as f:
+            f.write(json.dumps(line) + "\n")
+    except OSError:
+        pass
 
 TOL = {0: 1e-5, 1: 1e-12}  # fp32 / fp64 (north_star: ≤1e-5 fp32, ≤1e-12 fp64)
 
@@ -27,9 +49,18 @@ def gpu_run(prob, steps, precision, chunks=None):
     return out
 
 
-def errors(gpu, ora):
+def errors(gpu, ora, prec=None, steps=None, config=None):
     """(err_rho, err_u) normalised by the field maxima over all levels; also
-    checks the fluid-leaf sets agree."""
+    checks the fluid-leaf sets agree.  With prec given, the result is also
+    appended to the parity log (record)."""
+    er, eu = _errors(gpu, ora)
+    if prec is not None:
+        test = os.environ.get("PYTEST_CURRENT_TEST", "?").split(" ")[0]
+        record(test, str(config), int(steps or 0), prec, er, eu)
+    return er, eu
+
+
+def _errors(gpu, ora):
     dr = du = 0.0
     mr = mu = 0.0
     for (rg, ug), (ro, uo) in zip(gpu, ora):

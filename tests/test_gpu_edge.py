@@ -66,7 +66,7 @@ def test_level_without_fluid_leaves(prec):
     resolution): level 1 has nothing to update, level 0 bounces off it."""
     p = _random_state(_two_level((6, 5, 4), (slice(2, 4), slice(1, 3), slice(1, 3)), fine_code=2), 22)
     o = oracle_run(p, 6)
-    er, eu = errors(gpu_run(p, 6, prec), o)
+    er, eu = errors(gpu_run(p, 6, prec), o, prec, 6, p.name)
     assert er <= TOL[prec] and eu <= TOL[prec], (er, eu)
 
 
@@ -114,7 +114,7 @@ TINY = [((1, 1, 1), 1, (1, 1, 1)), ((2, 3, 1), 1, (1, 0, 1)), ((3, 2, 2), 2, (1,
 def test_domains_smaller_than_a_block(n, levels, periodic, prec):
     p = tiny_problem(n, levels, periodic)
     o = oracle_run(p, 5)
-    er, eu = errors(gpu_run(p, 5, prec), o)
+    er, eu = errors(gpu_run(p, 5, prec), o, prec, 5, p.name)
     assert er <= TOL[prec] and eu <= TOL[prec], (er, eu)
 
 
@@ -126,5 +126,5 @@ def test_refined_slab_thinner_than_a_block(Q, coll, prec):
     cells share blocks on both sides."""
     p = _random_state(_two_level((9, 4, 5), (slice(4, 5), slice(0, 4), slice(0, 5)), Q=Q, collision=coll), 24)
     o = oracle_run(p, 8)
-    er, eu = errors(gpu_run(p, 8, prec), o)
+    er, eu = errors(gpu_run(p, 8, prec), o, prec, 8, p.name)
     assert er <= TOL[prec] and eu <= TOL[prec], (er, eu)

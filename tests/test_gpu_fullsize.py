@@ -3,8 +3,12 @@ times (the fused kernels replayed from the CUDA graph), on sampled outputs.
 
 Dense per-level arrays do not fit at these sizes (cfg5's finest level alone
 has 1.13 G cells), so both sides are read through probes (lbm_probe /
-Oracle.probe) at seeded random fluid leaves of every level, after one coarse
-step.  cfg3 / cfg4 / cfg5 compare with the fp64 oracle run on the same full
+Oracle.probe) at seeded random fluid leaves of every level, after FIVE coarse
+steps (so interface, wall, inlet and outflow cells have left the uniform
+initial state).  Half of every level's samples are drawn from its *special*
+leaves — fluid leaves with a 26-neighbour that is not a same-level fluid leaf
+(refinement interface, BC leaf, domain face) — where all the non-trivial
+rules act; the other half uniformly from all fluid leaves.  cfg3 / cfg4 / cfg5 compare with the fp64 oracle run on the same full
 grid; cfg2 (512^3 periodic, too large for the oracle's dense maps) compares
 with the one-step result the oracle's own collision and equilibrium compute
 cell by cell.  Bars as everywhere: fp32 <= 1e-5, fp64 <= 1e-12 relative to
@@ -22,6 +26,45 @@ pytestmark = pytest.mark.gpu
 
 FP32, FP64 = 0, 1
 N_SAMPLE = 100_000  # per level
+N_STEPS = 5
+
+
+def _special(prob, L):
+    """Fluid leaves of level L with a 26-neighbour that is not a same-level
+    fluid leaf (outside the domain counts on non-periodic axes)."""
+    fluid = prob.masks[L] == 1
+    d = ~fluid
+    for ax in range(3):
+        a = d.copy()
+        if prob.periodic[ax]:
+            a |= np.roll(d, 1, ax)
+            a |= np.roll(d, -1, ax)
+        else:
+            lo = [slice(None)] * 3
+            hi = [slice(None)] * 3
+            lo[ax], hi[ax] = slice(1, None), slice(None, -1)
+            a[tuple(lo)] |= d[tuple(hi)]
+            a[tuple(hi)] |= d[tuple(lo)]
+            e0 = [slice(None)] * 3
+            e1 = [slice(None)] * 3
+            e0[ax], e1[ax] = 0, -1
+            a[tuple(e0)] = True
+            a[tuple(e1)] = True
+        d = a
+    return fluid & d
+
+
+def _sample_mixed(prob, L, n, seed):
+    """n/2 special leaves and n/2 uniform fluid leaves of level L (fewer if the
+    level has fewer)."""
+    m = prob.masks[L]
+    rng = np.random.default_rng(seed + 100 * L)
+    spec = np.flatnonzero(_special(prob, L))
+    flat = np.flatnonzero(m == 1)
+    a = rng.choice(spec, size=min(n // 2, spec.size), replace=False) if spec.size else np.zeros(0, np.int64)
+    b = rng.choice(flat, size=min(n - a.size, flat.size), replace=False)
+    pick = np.concatenate([a, b])
+    return np.stack(np.unravel_index(pick, m.shape), axis=1).astype(np.int64), a.size
 
 
 def _sample(prob, L, n, seed):
@@ -43,7 +86,7 @@ def _rel_err(gpu, ref):
     return dr / mr, du / max(mu, 1e-300)
 
 
-def _gpu_probe(prob, prec, samples, steps=1):
+def _gpu_probe(prob, prec, samples, steps=N_STEPS):
     from paper_conf_ipps_mahmoudsm24_b200 import lbmr
     g = lbmr.grid_from_problem(prob, precision=prec)
     g.step(steps)
@@ -61,16 +104,24 @@ FULL = {
 
 @pytest.mark.parametrize("name", list(FULL))
 def test_full_size_sampled_parity(name):
+    from tests._parity import record
     prob = FULL[name]()
-    samples = [_sample(prob, L, N_SAMPLE, 17) for L in range(prob.levels)]
+    mixed = [_sample_mixed(prob, L, N_SAMPLE, 17) for L in range(prob.levels)]
+    samples = [m[0] for m in mixed]
+    n_special = [m[1] for m in mixed]
+    # half of every level's sample is special (all of its special leaves when it has fewer)
+    for L in range(prob.levels):
+        assert n_special[L] == min(N_SAMPLE // 2, int(_special(prob, L).sum())), (L, n_special[L])
     o = oracle.Oracle(prob)
-    o.step(1)
+    o.step(N_STEPS)
     ref = [o.probe(L, xyz) for L, xyz in enumerate(samples)]
     del o
     gc.collect()
     for prec in (FP64, FP32):
         got = _gpu_probe(prob, prec, samples)
         er, eu = _rel_err(got, ref)
+        record("test_full_size_sampled_parity", name, N_STEPS, prec, er, eu,
+               samples=[len(s) for s in samples], special_samples=n_special)
         assert er <= TOL[prec] and eu <= TOL[prec], (name, prec, er, eu)
 
 
@@ -94,7 +145,7 @@ def test_full_size_uniform512_one_step():
         ref_r[k] = f.sum()
         ref_u[k] = (e * f[:, None]).sum(axis=0) / ref_r[k]
     for prec in (FP64, FP32):
-        got = _gpu_probe(prob, prec, [xyz])[0]
+        got = _gpu_probe(prob, prec, [xyz], steps=1)[0]
         er, eu = _rel_err([got], [(ref_r, ref_u)])
         assert er <= TOL[prec] and eu <= TOL[prec], (prec, er, eu)
 

@@ -1,5 +1,8 @@
 """Multi-GPU x-slab path on one device (T13): P partitions == one grid, bitwise
-in fp64 (the gather coalescence is deterministic and a halo cell is a copy).
+in fp64 (the gather coalescence is deterministic and a halo cell is a copy),
+and P partitions == the fp64 oracle within the parity bar (the partitioned
+result is checked against the oracle directly, not only against the
+single-grid CUDA run).
 
 * in one process: P slab grids on P streams, halos connected directly
   (`lbm_halo_connect_local`), the device-side flag protocol orders them;
@@ -13,6 +16,7 @@ import numpy as np
 import pytest
 
 import lbm_inputs as I
+from tests._parity import TOL, errors, oracle_run, record
 
 pytestmark = pytest.mark.gpu
 
@@ -37,6 +41,10 @@ CASES = [
     ("slab_periodic", lambda: I.planar_slab(levels=3, n=(16, 8, 8)), 3, 6),
     ("random_px", lambda: I.random_balanced(41, n=(12, 6, 6), levels=3, p_refine=0.6, periodic=(1, 0, 1)), 3, 5),
     ("kbc_mini", lambda: I.cavity4_kbc("mini"), 2, 3),
+    # 8 ranks on the reduced tunnel (40 coarse columns, 4 levels): the
+    # driver's 8-GPU run uses the same code path on the full cfg5
+    ("tunnel4_s5", lambda: I.tunnel4(scale=5), 8, 20),
+    ("random_px", lambda: I.random_balanced(41, n=(12, 6, 6), levels=3, p_refine=0.6, periodic=(1, 0, 1)), 8, 20),
 ]
 
 
@@ -47,30 +55,45 @@ def test_partitioned_equals_single_grid(name, mk, P, steps):
     ref = _single(prob, steps, FP64)
     pg = lbmr.PartitionedGrid(prob, P, precision=FP64)
     pg.step(steps)
+    got = []
     for L in range(prob.levels):
         r, u = pg.macroscopic(L)
+        got.append((r, u))
         assert np.array_equal(np.isnan(r), np.isnan(ref[L][0])), (name, L)
         m = ~np.isnan(r)
         assert np.array_equal(r[m], ref[L][0][m]), (name, L, np.abs(r[m] - ref[L][0][m]).max())
         assert np.array_equal(u[m], ref[L][1][m]), (name, L)
     pg.close()
+    # and directly against the oracle
+    er, eu = errors(got, oracle_run(prob, steps))
+    record(f"test_partitioned_equals_single_grid[{name}-P{P}]", name, steps, FP64, er, eu, ranks=P)
+    assert er <= TOL[FP64] and eu <= TOL[FP64], (name, P, er, eu)
 
 
-def test_partitioned_fp32_and_chunked_steps():
+@pytest.mark.parametrize("P", [3, 8])
+def test_partitioned_fp32_and_chunked_steps(P):
     from paper_conf_ipps_mahmoudsm24_b200 import lbmr
     prob = I.tunnel4(scale=5)
     ref = _single(prob, 5, FP32)
-    pg = lbmr.PartitionedGrid(prob, 3, precision=FP32)
+    pg = lbmr.PartitionedGrid(prob, P, precision=FP32)
     for n in (1, 3, 1):
         pg.step(n)
+    got = []
     for L in range(prob.levels):
         r, u = pg.macroscopic(L)
+        got.append((r, u))
         m = ~np.isnan(r)
         assert np.array_equal(r[m], ref[L][0][m]) and np.array_equal(u[m], ref[L][1][m])
     pg.close()
+    er, eu = errors(got, oracle_run(prob, 5))
+    record(f"test_partitioned_fp32_and_chunked_steps[P{P}]", "tunnel4_s5", 5, FP32, er, eu, ranks=P)
+    assert er <= TOL[FP32] and eu <= TOL[FP32], (P, er, eu)
 
 
-def _ipc_worker(rank, world, port, steps, q):
+IPC_PROBLEMS = {"cavity2": lambda: I.cavity2("r"), "tunnel4_s5": lambda: I.tunnel4(scale=5)}
+
+
+def _ipc_worker(rank, world, port, steps, q, pname="cavity2"):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     import torch
@@ -79,7 +102,7 @@ def _ipc_worker(rank, world, port, steps, q):
     try:
         from paper_conf_ipps_mahmoudsm24_b200 import lbmr
         torch.cuda.set_device(0)
-        prob = I.cavity2("r")
+        prob = IPC_PROBLEMS[pname]()
         s = torch.cuda.Stream()
         g = lbmr.grid_from_problem(prob, FP64, stream=s.cuda_stream, n_ranks=world, rank=rank)
         blobs = {}
@@ -104,9 +127,11 @@ def _ipc_worker(rank, world, port, steps, q):
         dist.destroy_process_group()
 
 
-def test_two_processes_cuda_ipc_halo():
-    """Two processes on the same GPU, halos written into the neighbour's
-    buffers through CUDA IPC + the device flag protocol (the 8xB200 path)."""
+@pytest.mark.parametrize("world,pname,steps", [(2, "cavity2", 4), (8, "tunnel4_s5", 6)])
+def test_processes_cuda_ipc_halo(world, pname, steps):
+    """`world` processes on the same GPU, halos written into the neighbour's
+    buffers through CUDA IPC + the device flag protocol (the 8xB200 path):
+    bitwise equal to one grid, and within the fp64 bar of the oracle."""
     import torch.multiprocessing as mp
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
@@ -114,19 +139,25 @@ def test_two_processes_cuda_ipc_halo():
     s.bind(("127.0.0.1", 0))
     port = s.getsockname()[1]
     s.close()
-    steps = 4
-    procs = [ctx.Process(target=_ipc_worker, args=(r, 2, port, steps, q)) for r in range(2)]
+    procs = [ctx.Process(target=_ipc_worker, args=(r, world, port, steps, q, pname)) for r in range(world)]
     for p in procs:
         p.start()
-    res = dict(q.get(timeout=600) for _ in range(2))
+    res = dict(q.get(timeout=900) for _ in range(world))
     for p in procs:
         p.join(timeout=120)
-    for r in range(2):
+    for r in range(world):
         assert not isinstance(res[r], str), res[r]
-    prob = I.cavity2("r")
+    prob = IPC_PROBLEMS[pname]()
     ref = _single(prob, steps, FP64)
+    got = []
     for L in range(prob.levels):
-        r = np.concatenate([res[0][L][0], res[1][L][0]], axis=0)
+        r = np.concatenate([res[k][L][0] for k in range(world)], axis=0)
+        u = np.concatenate([res[k][L][1] for k in range(world)], axis=0)
+        got.append((r, u))
         m = ~np.isnan(r)
         assert np.array_equal(m, ~np.isnan(ref[L][0]))
         assert np.array_equal(r[m], ref[L][0][m])
+        assert np.array_equal(u[m], ref[L][1][m])
+    er, eu = errors(got, oracle_run(prob, steps))
+    record(f"test_processes_cuda_ipc_halo[{world}-{pname}]", pname, steps, FP64, er, eu, ranks=world, transport="cuda_ipc")
+    assert er <= TOL[FP64] and eu <= TOL[FP64], (er, eu)

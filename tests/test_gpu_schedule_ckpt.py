@@ -66,7 +66,7 @@ def test_unfused_matches_oracle():
     prob = I.cavity2("r")
     ora = oracle_run(prob, 10)
     for prec in (FP64, FP32):
-        er, eu = errors(_run(prob, prec, 10, lbmr.SCHED_UNFUSED), ora)
+        er, eu = errors(_run(prob, prec, 10, lbmr.SCHED_UNFUSED), ora, prec, 10, "cavity2r/unfused")
         assert er <= TOL[prec] and eu <= TOL[prec], (prec, er, eu)
 
 
@@ -86,8 +86,9 @@ def test_schedule_switch_mid_run():
 def test_bad_schedule_mode():
     lbmr = _lbmr()
     g = lbmr.grid_from_problem(I.cavity2(), precision=FP32)
-    with pytest.raises(lbmr.LBMError):
-        g.set_schedule(7)
+    for bad in (64, -1, lbmr.SCHED_SPLIT_A | lbmr.SCHED_ATOMIC_A):
+        with pytest.raises(lbmr.LBMError):
+            g.set_schedule(bad)
     g.close()
 
 
@@ -154,6 +155,52 @@ def test_checkpoint_partitioned_bitwise():
     got = [pg2.macroscopic(L) for L in range(prob.levels)]
     pg2.close()
     _same(ref, got)
+
+
+def test_checkpoint_partitioned_without_global_sync():
+    """lbm_checkpoint_save on one slab must itself wait for the
+    neighbour's final halo stores into its buffers (no caller-side global
+    synchronisation before saving).  Slabs are saved right after the steps
+    are issued, slab 0 first (its neighbour's kernels may still be running)."""
+    lbmr = _lbmr()
+    prob = I.tunnel4(scale=5)
+    ref = _run(prob, FP64, 6, lbmr.SCHED_FUSED)
+    for P in (2, 4):
+        pg = lbmr.PartitionedGrid(prob, P, precision=FP64)
+        pg.step(3)
+        cks = [g.save_checkpoint() for g in pg.grids]
+        pg.close()
+        pg2 = lbmr.PartitionedGrid(prob, P, precision=FP64)
+        for g, ck in zip(pg2.grids, cks):
+            g.load_checkpoint(ck)
+        pg2.step(3)
+        got = [pg2.macroscopic(L) for L in range(prob.levels)]
+        pg2.close()
+        _same(ref, got)
+
+
+def test_device_bytes_and_launch_count_match_analyze():
+    """lbm_grid_analyze predicts exactly the device bytes lbm_grid_create
+    allocates and the kernels one coarse step launches."""
+    lbmr = _lbmr()
+    for prob in (I.tunnel4(scale=5), I.cavity4_kbc("mini"), I.cavity2()):
+        for prec in (FP32, FP64):
+            a = lbmr.analyze_problem(prob, precision=prec)
+            g = lbmr.grid_from_problem(prob, precision=prec, init=False)
+            i = g.info()
+            assert i.device_bytes == a.device_bytes, (prob.name, prec, i.device_bytes, a.device_bytes)
+            assert i.launches_per_step == a.launches_per_step
+            g.close()
+    prob = I.tunnel4(scale=5)
+    pg = lbmr.PartitionedGrid(prob, 2, precision=FP32)
+    for r, g in enumerate(pg.grids):
+        a = lbmr.analyze(prob.nx, prob.ny, prob.nz, prob.masks, n_ranks=2, rank=r, **lbmr._problem_kw(prob, FP32))
+        i = g.info()
+        assert i.device_bytes >= a.device_bytes  # + the peer cell lists uploaded at connect
+        # one halo wait per level kernel and per coalescence gather
+        assert i.launches_per_step == a.launches_per_step
+        assert i.launches_per_step > i.kernels_per_step * 2
+    pg.close()
 
 
 @pytest.mark.parametrize("prec", [0, 1])

@@ -62,7 +62,7 @@ def test_volumetric_matches_oracle(name, prec):
     steps = STEPS.get(name, 5)
     if name not in _cache:
         _cache[name] = _oracle_vol(prob, steps)
-    er, eu = errors(_gpu_vol(prob, prec, steps), _cache[name])
+    er, eu = errors(_gpu_vol(prob, prec, steps), _cache[name], prec, steps, name + "/volumetric")
     assert er <= TOL[prec] and eu <= TOL[prec], (name, prec, er, eu)
 
 
