@@ -49,7 +49,10 @@ for _s in (1, 2, 3):
 DEFAULT_PRECISION = {f"sphere_tab1_s{_s}": "fp64" for _s in (1, 2, 3)}
 # the paper's own number for exactly this metric and workload (A100, fp64), Tab. I
 PAPER_MLUPS = {f"sphere_tab1_s{_s}": I.TAB1[_s]["ours_mlups"] for _s in (1, 2, 3)}
-SCHEDULES = {"fused": 0, "unfused": 1, "nograph": 2, "unfused_nograph": 3}
+# lbm_set_schedule bit sets (lbmr.h): the product, the C/S split, the graph-free
+# launch path, and the paper's Fig. 4 fusion configurations (lbmr.FIG4)
+SCHEDULES = {"fused": 0, "unfused": 1, "nograph": 2, "unfused_nograph": 3,
+             "fig4b": 1 | 4 | 8 | 32, "fig4c": 1 | 4 | 16 | 32, "fig4d": 1 | 8 | 32, "fig4e": 1 | 16, "fig4f": 16}
 N_PROBE = 4096  # e2e monitoring cells
 # bounded oracle sample for --impl reference (one coarse step per timed step)
 REF_SAMPLE = {
@@ -366,9 +369,7 @@ def main():
         torch.distributed.all_reduce(t)
         leaves = [int(v) for v in t.tolist()]
     upd = updates_per_step(leaves)
-    launches_per_step = int(info.launches_per_step)
-    if SCHEDULES[args.schedule] & 1:  # unfused: stream + collide kernel per level-substep
-        launches_per_step += int(info.kernels_per_step)
+    launches_per_step = int(info.launches_per_step)  # for the schedule set above (lbm_grid_get_info)
 
     g.step(args.warmup)
     g.synchronize()

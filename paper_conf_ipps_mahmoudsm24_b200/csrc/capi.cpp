@@ -100,6 +100,8 @@ struct lbm_grid {
   bool broken = false;
   int sched = LBM_SCHED_FUSED;  // lbm_set_schedule
   bool pdl = true;              // programmatic dependent launch of F_L^k after its gather (LBMR_NO_PDL=1: off)
+  bool peer_other_gpu[2] = {false, false};  // the connected neighbour on this side is on another GPU
+  bool halo_spin = false;       // in-kernel halo waits (every connected neighbour on another GPU)
   int64_t steps = 0;
   int64_t device_bytes = 0;
   std::vector<void*> allocs;
@@ -243,6 +245,7 @@ StepParams<T> make_params(const lbm_grid* g, int L, int64_t k) {
   if (g->n_ranks > 1) {
     const HostLevel& H = g->host[L];
     p.nbctas = std::max(kHaloCtasPerBlock * H.nboundary, 1);
+    p.halo_spin = g->halo_spin ? 1 : 0;
     p.nboundary = H.nboundary;
     p.flags = g->flags;
     p.bpeer = D.bpeer;
@@ -280,8 +283,19 @@ bool level_has_coal(const lbm_grid* g, int L) {
 
 void launch_gather(lbm_grid* g, int L, const void* fa, const void* fb, void* dst, int mode) {
   const HostLevel& H = g->host[L];
+  const bool spin = g->n_ranks > 1 && g->halo_spin;
   launch_coalesce(g->Q, g->prec, fa, fb, dst, g->dev[L].coal_fill, g->dev[L].coal_cand, H.coal_n[0], H.coal_n[1], mode,
-                  g->stream);
+                  g->stream, spin ? g->flags : nullptr, g->has_nb[0], g->has_nb[1]);
+}
+
+// In-kernel halo waits when every connected neighbour is on another GPU
+// (LBMR_HALO_SPIN=1 / 0 forces them on / off).
+void update_halo_spin(lbm_grid* g) {
+  bool all = true;
+  for (int sd = 0; sd < 2; ++sd)
+    if (g->has_nb[sd] && !(g->connected[sd] && g->peer_other_gpu[sd])) all = false;
+  if (const char* e = getenv("LBMR_HALO_SPIN")) all = e[0] == '1';
+  g->halo_spin = all;
 }
 
 // ablation fields of the level-L launch producing C_L^{k+1} (k = 0: prologue)
@@ -346,7 +360,7 @@ void launch_F_typed(lbm_grid* g, int L, int64_t k, int kind, cudaEvent_t mid = n
                 g->dev[L + 1].pop[1], g->dev[L + 1].pop[0], g->bc_dev, g->face_dev, g->dev[L].vtemp, g->stream);
   // coalescence ghosts of C_L^k from C_{L+1}^{2k-1} and C_{L+1}^{2k} (both ready now)
   if (level_has_coal(g, L)) {
-    if (g->n_ranks > 1) {
+    if (g->n_ranks > 1 && !g->halo_spin) {
       // the gather reads L+1 halo cells: it follows the neighbour wait of F_L^k,
       // which launch_level_step issues first; issue an explicit wait here instead
       launch_halo_wait(p.flags, p.has_nb[0], p.has_nb[1], g->stream);
@@ -648,7 +662,8 @@ static int64_t planned_device_bytes(const std::vector<HostLevel>& host, int Q, s
   return t;
 }
 
-static void fill_info(const std::vector<HostLevel>& host, int Q, int prec, int n_ranks, lbm_grid_info* info) {
+static void fill_info(const std::vector<HostLevel>& host, int Q, int prec, int n_ranks, lbm_grid_info* info,
+                      int sched = 0, bool halo_spin = false) {
   std::memset(info, 0, sizeof(*info));
   info->levels = (int32_t)host.size();
   info->Q = Q;
@@ -656,11 +671,21 @@ static void fill_info(const std::vector<HostLevel>& host, int Q, int prec, int n
   info->kernels_per_step = (1 << host.size()) - 1;
   info->launches_per_step = info->kernels_per_step;
   // partitioned grid: a one-thread halo wait before every level kernel
-  if (n_ranks > 1) info->launches_per_step += info->kernels_per_step;
+  // (unless the waits are in-kernel: neighbours on other GPUs)
+  const bool waits = n_ranks > 1 && !halo_spin;
+  if (waits) info->launches_per_step += info->kernels_per_step;
   for (size_t L = 0; L < host.size(); ++L) {
     // the coalescence gather before every F_L^k (and its own halo wait when partitioned)
-    if (!host[L].coal_fill.empty()) info->launches_per_step += ((int64_t)1 << L) * (n_ranks > 1 ? 2 : 1);
+    if (!host[L].coal_fill.empty()) info->launches_per_step += ((int64_t)1 << L) * (waits ? 2 : 1);
     if (!host[L].vavg.empty()) info->launches_per_step += (int64_t)2 << L;
+    // ablation schedules (lbm_set_schedule): split kernels per level-substep
+    const int64_t sub = (int64_t)1 << L;
+    const bool coal = L + 1 < (int)host.size() && !host[L].coal_fill.empty();
+    if (sched & LBM_SCHED_UNFUSED) info->launches_per_step += sub;  // S and C
+    if (coal && (sched & (LBM_SCHED_SPLIT_A | LBM_SCHED_ATOMIC_A))) info->launches_per_step -= sub;  // no gather
+    if (coal && (sched & LBM_SCHED_SPLIT_A)) info->launches_per_step += sub * 2;  // A after each fine substep
+    if (coal && (sched & LBM_SCHED_SPLIT_O)) info->launches_per_step += sub;  // O
+    if ((sched & LBM_SCHED_SPLIT_E) && L > 0 && !host[L].ghost_fill.empty()) info->launches_per_step += sub;  // E
     info->leaves[L] = host[L].leaves;
     for (int a = 0; a < 3; ++a) info->block_offset[L][a] = host[L].off[a];
     info->blocks[L] = host[L].nfluid;
@@ -1362,7 +1387,7 @@ lbm_status lbm_stats(lbm_grid* g, int64_t* leaves, double* mass) {
 lbm_status lbm_grid_get_info(const lbm_grid* g, lbm_grid_info* info) {
   g_err.clear();
   if (!g || !info) return fail(LBM_E_INVAL, "NULL argument");
-  fill_info(g->host, g->Q, g->prec, g->n_ranks, info);
+  fill_info(g->host, g->Q, g->prec, g->n_ranks, info, g->sched, g->halo_spin);
   info->device_bytes = g->device_bytes;
   info->steps_done = g->steps;
   return LBM_OK;
@@ -1396,6 +1421,7 @@ struct HaloBlob {
   uint32_t magic, version;
   int32_t levels, Q, prec, side, rank, n_ranks;
   int32_t pid, device;
+  char pci[32];  // PCI bus id of the exporter's GPU (same physical GPU -> halo_wait kernels)
   int64_t count[16];
   cudaIpcMemHandle_t pop[16][2];
   cudaIpcMemHandle_t flags;
@@ -1447,6 +1473,7 @@ lbm_status lbm_halo_export(const lbm_grid* g, int32_t side, void* blob, int64_t 
   h.n_ranks = g->n_ranks;
   h.pid = (int32_t)getpid();
   cudaGetDevice(&h.device);
+  cudaDeviceGetPCIBusId(h.pci, (int)sizeof(h.pci), h.device);
   for (int L = 0; L < g->levels; ++L) {
     h.count[L] = (int64_t)g->host[L].halo[side].size();
     for (int b = 0; b < 2; ++b) CUDA_TRY(cudaIpcGetMemHandle(&h.pop[L][b], g->dev[L].pop[b]));
@@ -1502,11 +1529,17 @@ lbm_status lbm_halo_connect(lbm_grid* g, int32_t side, const void* blob, int64_t
   void* f = nullptr;
   if ((s = open_ipc(g, h.flags, &f))) return s;
   g->peer_flags[side] = static_cast<unsigned long long*>(f);
+  {
+    char mine[32] = {0};
+    cudaDeviceGetPCIBusId(mine, (int)sizeof(mine), g->device);
+    g->peer_other_gpu[side] = std::strncmp(mine, h.pci, sizeof(mine)) != 0;
+  }
   // every local write to the buffers the peer stores into (zero-fill, init)
   // is complete before the caller's barrier lets the peer start stepping
   CUDA_TRY(cudaStreamSynchronize(g->stream));
   CUDA_TRY(cudaDeviceSynchronize());
   g->connected[side] = true;
+  update_halo_spin(g);
   return LBM_OK;
 }
 
@@ -1542,6 +1575,8 @@ lbm_status lbm_halo_connect_local(lbm_grid* g, int32_t side, lbm_grid* peer) {
   CUDA_TRY(cudaStreamSynchronize(g->stream));
   CUDA_TRY(cudaStreamSynchronize(peer->stream));
   g->connected[side] = true;
+  g->peer_other_gpu[side] = peer->device != g->device;
+  update_halo_spin(g);
   return LBM_OK;
 }
 

@@ -80,6 +80,7 @@ struct StepParams {
   int32_t nbctas;               // CTAs taking part in the halo protocol (cut-plane blocks, >= 1)
   int32_t nboundary;            // cut-plane blocks (stored and launched first)
   int32_t has_nb[2];            // neighbour on the -x / +x side
+  int32_t halo_spin;            // 1: protocol CTAs wait in-kernel (neighbours on other GPUs), 0: halo_wait_kernel
   unsigned long long* flags;    // this rank: [0],[1] bumped by the -x/+x neighbour, [2] kernels done, [3] CTA count
   unsigned long long* peer_flag[2];  // neighbour's flag slot this rank bumps
   T* peer_dst[2];               // neighbour's C_L^{k+1} buffer
@@ -98,8 +99,11 @@ struct StepParams {
 // ablation schedules split it into Accumulate (fa or fb only, no division)
 // and Coalescence O (no source, kCoalFromDst | kCoalDivide) kernels.
 enum { kCoalFromDst = 1, kCoalDivide = 2 };
+// spin_flags (partitioned grid whose neighbours are on other GPUs): every CTA
+// first waits in-kernel for the neighbours' previous kernels (halo protocol).
 void launch_coalesce(int Q, int precision, const void* fa, const void* fb, void* dst, const uint32_t* fill,
-                     const uint32_t* cand, int64_t n_main, int64_t n_ovf, int mode, cudaStream_t s);
+                     const uint32_t* cand, int64_t n_main, int64_t n_ovf, int mode, cudaStream_t s,
+                     const unsigned long long* spin_flags = nullptr, int nb0 = 0, int nb1 = 0);
 
 // rho / u (double) of n cells given by population cell index block*512+local
 // (-1 -> NaN), read from the post-collision buffer `pop`.

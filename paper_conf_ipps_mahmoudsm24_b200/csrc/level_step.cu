@@ -87,6 +87,9 @@ __host__ __device__ constexpr int wclass(int q) { return q == 0 ? 0 : q < 7 ? 1 
 // pairs (q, q+1):  ω g^eq_q = A_w + B_w (e_q.j) + C_w (e_q.j)^2 with
 //   A_w = ω w (δρ - 1.5 |j|^2/ρ),  B_w = 3 ω w,  C_w = 4.5 ω w / ρ
 // (ρ u = j), so the pair shares A + C (e.j)^2 and flips the sign of B (e.j).
+#ifndef LBMR_BGK_ALT_FORM
+#define LBMR_BGK_ALT_FORM 0
+#endif
 template <int Q, typename T>
 __device__ __forceinline__ void collide_bgk(T (&g)[Q], T omega) {
   T drho = g[0], jx = T(0), jy = T(0), jz = T(0);
@@ -113,6 +116,26 @@ __device__ __forceinline__ void collide_bgk(T (&g)[Q], T omega) {
     B[c] = w * bfac;
     C[c] = w * cfac;
   }
+#if LBMR_BGK_ALT_FORM
+  // diagnostic build only (tools/fp32_floor.py): the same BGK step in another
+  // association, g* = g - ω (g - g^eq), to measure how far two equally valid
+  // fp32 evaluations of the method drift apart
+  (void)omw;
+  const T iw = recip<T>(omega);
+  g[0] = g[0] - omega * (g[0] - A[0] * iw);
+#pragma unroll
+  for (int q = 1; q < Q; q += 2) {
+    T ej = T(0);
+    if (ex(q) > 0) ej += jx; else if (ex(q) < 0) ej -= jx;
+    if (ey(q) > 0) ej += jy; else if (ey(q) < 0) ej -= jy;
+    if (ez(q) > 0) ej += jz; else if (ez(q) < 0) ej -= jz;
+    const int c = wclass(q);
+    const T sym = (C[c] * ej * ej + A[c]) * iw;
+    const T asym = B[c] * ej * iw;
+    g[q] = g[q] - omega * (g[q] - (sym + asym));
+    g[q + 1] = g[q + 1] - omega * (g[q + 1] - (sym - asym));
+  }
+#else
   g[0] = omw * g[0] + A[0];
 #pragma unroll
   for (int q = 1; q < Q; q += 2) {
@@ -126,6 +149,7 @@ __device__ __forceinline__ void collide_bgk(T (&g)[Q], T omega) {
     g[q] = omw * g[q] + (sym + asym);
     g[q + 1] = omw * g[q + 1] + (sym - asym);
   }
+#endif
 }
 
 template <>
@@ -895,7 +919,7 @@ __device__ __forceinline__ unsigned long long globaltimer_ns() {
   return t;
 }
 
-__global__ void halo_wait_kernel(const unsigned long long* flags, int nb0, int nb1) {
+__device__ __forceinline__ void halo_spin_wait(const unsigned long long* flags, int nb0, int nb1) {
   const unsigned long long mine = *(volatile const unsigned long long*)(flags + 2);
   const unsigned long long t0 = globaltimer_ns();
   for (int s = 0; s < 2; ++s) {
@@ -910,6 +934,22 @@ __global__ void halo_wait_kernel(const unsigned long long* flags, int nb0, int n
   }
 }
 
+__global__ void halo_wait_kernel(const unsigned long long* flags, int nb0, int nb1) {
+  halo_spin_wait(flags, nb0, nb1);
+}
+
+// In-kernel form (P.halo_spin, set when every neighbour rank is on another
+// GPU): only the CTAs that read halo cells or store into the neighbour (the
+// protocol CTAs) wait, thread 0 spinning and the CTA's barrier ordering the
+// other threads' reads after its acquire.  Saves the one-thread wait kernel
+// and its graph-node gap before every level kernel.  Not used when ranks
+// share a GPU: there, spinning CTAs could hold every SM slot while the kernel
+// they wait for has none.
+__device__ __forceinline__ void halo_spin_cta(const unsigned long long* flags, int nb0, int nb1) {
+  if (threadIdx.x == 0) halo_spin_wait(flags, nb0, nb1);
+  __syncthreads();
+}
+
 template <int Q, int COLL, typename T, bool STREAM>
 __global__ void __launch_bounds__(kHaloCtaThreads, (PlainOcc<Q, T, COLL>::value * 256) / kHaloCtaThreads)
     level_step_halo(const StepParams<T> P) {
@@ -922,6 +962,7 @@ __global__ void __launch_bounds__(kHaloCtaThreads, (PlainOcc<Q, T, COLL>::value 
   // read L-1 halo cells) count towards this kernel's completion signal
   const bool fill = (int)blockIdx.x >= main;
   const bool proto = (int)blockIdx.x < P.nbctas || fill;
+  if (P.halo_spin && proto) halo_spin_cta(P.flags, P.has_nb[0], P.has_nb[1]);
   if (fill) {
     trail_fill<Q, T>(P, ((int)blockIdx.x - main) * NT + threadIdx.x);
   } else if (blk < P.nfluid) {
@@ -1110,8 +1151,12 @@ template <typename T>
 __global__ void __launch_bounds__(256) coalesce_kernel(const T* __restrict__ fa, const T* __restrict__ fb, T* dst,
                                                        const uint32_t* __restrict__ fill,
                                                        const uint32_t* __restrict__ cand, int64_t nmain, int64_t novf,
-                                                       int mode) {
+                                                       int mode, const unsigned long long* spin_flags, int nb0,
+                                                       int nb1) {
   pdl_launch_dependents();  // the level kernel after it may start (it waits where it needs us)
+  // partitioned grid on distinct GPUs: the candidates may be halo cells of the
+  // finer level, written by the neighbour's last fine kernel
+  if (spin_flags) halo_spin_cta(spin_flags, nb0, nb1);
   const int64_t i = (int64_t)blockIdx.x * 256 + threadIdx.x;
   if (i < nmain) {
     coalesce_one<T, kCoalSlots>(fa, fb, dst, __ldg(fill + i), cand + i, nmain, mode);
@@ -1182,17 +1227,18 @@ void launch_halo_wait(const unsigned long long* flags, int nb0, int nb1, cudaStr
 }
 
 void launch_coalesce(int Q, int precision, const void* fa, const void* fb, void* dst, const uint32_t* fill,
-                     const uint32_t* cand, int64_t n_main, int64_t n_ovf, int mode, cudaStream_t s) {
+                     const uint32_t* cand, int64_t n_main, int64_t n_ovf, int mode, cudaStream_t s,
+                     const unsigned long long* spin_flags, int nb0, int nb1) {
   (void)Q;
   const int64_t n = n_main + n_ovf;
   if (n <= 0) return;
   const unsigned grid = (unsigned)((n + 255) / 256);
   if (precision == LBM_FP32)
     coalesce_kernel<float><<<grid, 256, 0, s>>>((const float*)fa, (const float*)fb, (float*)dst, fill, cand, n_main,
-                                                 n_ovf, mode);
+                                                 n_ovf, mode, spin_flags, nb0, nb1);
   else
     coalesce_kernel<double><<<grid, 256, 0, s>>>((const double*)fa, (const double*)fb, (double*)dst, fill, cand,
-                                                  n_main, n_ovf, mode);
+                                                  n_main, n_ovf, mode, spin_flags, nb0, nb1);
 }
 
 // ---------------------------------------------------------------- dispatch
@@ -1212,7 +1258,7 @@ static void launch_typed(int kind, const void* params, cudaStream_t s) {
     return;
   }
   if (p.nbctas > 0) {  // partitioned: always launched (the protocol must run)
-    halo_wait_kernel<<<1, 1, 0, s>>>(p.flags, p.has_nb[0], p.has_nb[1]);
+    if (!p.halo_spin) halo_wait_kernel<<<1, 1, 0, s>>>(p.flags, p.has_nb[0], p.has_nb[1]);
     dim3 grid(kHaloCtasPerBlock * std::max(p.nfluid, 1) + halo_fill_ctas(trail_count(p)));
     const size_t hs = (size_t)Q * kHaloCtaThreads * sizeof(T);
     if (kind == 1) level_step_halo<Q, COLL, T, false><<<grid, dim3(kHaloCtaThreads), 0, s>>>(p);

@@ -16,12 +16,13 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 PARITY_LOG = os.environ.get("LBMR_PARITY_LOG", os.path.join(ROOT, "gpurun_out", "parity_errors.jsonl"))
 
 
-def record(test: str, config: str, steps: int, precision: int, err_rho: float, err_u: float, **extra):
+def record(test: str, config: str, steps: int, precision: int, err_rho: float, err_u: float, bar=None, **extra):
     """Append one measured (err_rho, err_u) to the parity log (best effort)."""
     try:
         os.makedirs(os.path.dirname(PARITY_LOG), exist_ok=True)
         line = {"test": test, "config": config, "steps": int(steps), "precision": "fp64" if precision else "fp32",
-                "err_rho": float(err_rho), "err_u": float(err_u), "bar": TOL[precision], "time": time.time(), **extra}
+                "err_rho": float(err_rho), "err_u": float(err_u), "bar": float(bar if bar is not None else TOL[precision]),
+                "time": time.time(), **extra}
         with open(PARITY_LOG, "a") as f:
             f.write(json.dumps(line) + "\n")
     except OSError:
@@ -74,3 +75,21 @@ def _errors(gpu, ora):
         mr = max(mr, np.abs(ro[mo]).max())
         mu = max(mu, np.abs(uo[mo]).max())
     return dr / mr, (du / mu if mu > 0 else du)
+
+
+def rounding_drift(prob, steps, eps=4e-16, seed=7):
+    """The problem's own sensitivity to rounding (reading R-B4): the
+    (err_rho, err_u) between the oracle run on `prob` and the oracle run on
+    the same problem whose initial density carries a relative perturbation of
+    `eps` (2 ulps of 1.0 in fp64), after `steps` coarse steps.  Two fp64
+    implementations of the same rules cannot be expected to agree more
+    closely than this."""
+    import dataclasses
+    rng = np.random.default_rng(seed)
+    p = dataclasses.replace(prob)
+    p.init_rho, p.init_u = [], []
+    for L in range(prob.levels):
+        r, u = prob.init_fields(L)
+        p.init_rho.append(r * (1 + eps * rng.uniform(-1, 1, r.shape)))
+        p.init_u.append(u)
+    return _errors(oracle_run(p, steps), oracle_run(prob, steps))

@@ -161,3 +161,36 @@ def test_processes_cuda_ipc_halo(world, pname, steps):
     er, eu = errors(got, oracle_run(prob, steps))
     record(f"test_processes_cuda_ipc_halo[{world}-{pname}]", pname, steps, FP64, er, eu, ranks=world, transport="cuda_ipc")
     assert er <= TOL[FP64] and eu <= TOL[FP64], (er, eu)
+
+
+@pytest.mark.parametrize("name,mk,P,steps", [
+    ("tunnel4_s5", lambda: I.tunnel4(scale=5), 2, 6),
+    ("cavity2", lambda: I.cavity2("r"), 3, 6),
+    ("slab_periodic", lambda: I.planar_slab(levels=3, n=(16, 8, 8)), 2, 6),
+], ids=["tunnel4_s5-P2", "cavity2-P3", "slab-P2"])
+def test_in_kernel_halo_spin_equals_single_grid(name, mk, P, steps, monkeypatch):
+    """The in-kernel form of the halo wait (protocol CTAs spin; used when every
+    neighbour rank is on another GPU, i.e. the 8xB200 runs) forced on one
+    device: bitwise equal to one grid, and no halo_wait launches."""
+    from paper_conf_ipps_mahmoudsm24_b200 import lbmr
+    monkeypatch.setenv("LBMR_HALO_SPIN", "1")
+    prob = mk()
+    ref = _single(prob, steps, FP64)
+    pg = lbmr.PartitionedGrid(prob, P, precision=FP64)
+    for g in pg.grids:
+        i = g.info()
+        a = lbmr.analyze(prob.nx, prob.ny, prob.nz, prob.masks, n_ranks=P, rank=0, **lbmr._problem_kw(prob, FP64))
+        assert i.launches_per_step < a.launches_per_step  # the wait kernels are gone
+    pg.step(steps)
+    for L in range(prob.levels):
+        r, u = pg.macroscopic(L)
+        m = ~np.isnan(r)
+        assert np.array_equal(m, ~np.isnan(ref[L][0]))
+        assert np.array_equal(r[m], ref[L][0][m]) and np.array_equal(u[m], ref[L][1][m]), (name, L)
+    pg.close()
+
+
+def test_processes_in_kernel_halo_spin(monkeypatch):
+    """Two processes (CUDA IPC) with the in-kernel halo wait forced on."""
+    monkeypatch.setenv("LBMR_HALO_SPIN", "1")
+    test_processes_cuda_ipc_halo(2, "cavity2", 4)
