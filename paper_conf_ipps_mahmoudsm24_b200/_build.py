@@ -53,5 +53,19 @@ def build(force: bool = False, verbose: bool = False, out: str = None, defines=(
     return lib
 
 
+ALT_LIB = os.path.join(LIBDIR, "liblbmr_alt.so")
+
+
+def build_alt(force: bool = False) -> str:
+    """Diagnostic build for the fp32 rounding-floor checks (tools/fp32_floor.py,
+    tests/test_gpu_parity.py): the same sources with the BGK step evaluated
+    in another, equally valid association (LBMR_BGK_ALT_FORM=1).  Never loaded
+    by the product path."""
+    if force or not os.path.exists(ALT_LIB) or os.path.getmtime(ALT_LIB) < os.path.getmtime(LIB):
+        build(out=ALT_LIB, defines=["LBMR_BGK_ALT_FORM=1"])
+    return ALT_LIB
+
+
 if __name__ == "__main__":
     print(build(force=True, verbose=True))
+    print(build_alt(force=True))

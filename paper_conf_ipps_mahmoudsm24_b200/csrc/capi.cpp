@@ -624,7 +624,8 @@ static lbm_status build_host(const lbm_grid_desc* d, int32_t levels, const uint8
   in.masks = masks;
   in.variant = d->variant;
   in.align_blocks = getenv("LBMR_NO_BLOCK_ALIGN") ? 0 : 1;  // A/B switch for measurements
-  if (const char* o = getenv("LBMR_BLOCK_ORDER")) in.block_order = std::strcmp(o, "raster") == 0 ? 1 : 0;
+  if (const char* o = getenv("LBMR_BLOCK_ORDER"))
+    in.block_order = std::strcmp(o, "raster") == 0 ? 1 : std::strcmp(o, "hilbert") == 0 ? 2 : 0;
   if (slab) {
     in.n0[0] = slab->desc.nx;
     in.periodic[0] = 0;

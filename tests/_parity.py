@@ -93,3 +93,26 @@ def rounding_drift(prob, steps, eps=4e-16, seed=7):
         p.init_rho.append(r * (1 + eps * rng.uniform(-1, 1, r.shape)))
         p.init_u.append(u)
     return _errors(oracle_run(p, steps), oracle_run(prob, steps))
+
+
+def fp32_rounding_floor(name, steps, got):
+    """fp32 rounding floor (reading R-B5): the CUDA fp32 result `got`
+    of problem `name` (tools/parity_growth.PROBLEMS) against the same step
+    computed by the diagnostic build liblbmr_alt.so, whose BGK step is the
+    same formula in another association (g - ω (g - g^eq) instead of
+    (1 - ω) g + ω g^eq).  Two equally valid fp32 evaluations differing by X
+    bound how close any fp32 implementation can stay to the exact (fp64)
+    trajectory.  Returns (err_rho, err_u) between the two."""
+    import subprocess
+    import sys
+    import tempfile
+    lib = os.path.join(ROOT, "paper_conf_ipps_mahmoudsm24_b200", "_lib", "liblbmr_alt.so")
+    if not os.path.exists(lib):
+        from paper_conf_ipps_mahmoudsm24_b200 import _build
+        _build.build_alt()
+    out = os.path.join(tempfile.mkdtemp(), "alt.npz")
+    subprocess.check_call([sys.executable, os.path.join(ROOT, "tools", "fp32_floor.py"), "--child", name, str(steps),
+                           out], env=dict(os.environ, LBMR_LIB=lib), cwd=ROOT)
+    z = np.load(out)
+    alt = [(z[f"{steps}_{L}_r"], z[f"{steps}_{L}_u"]) for L in range(len(got))]
+    return _errors(got, alt)
