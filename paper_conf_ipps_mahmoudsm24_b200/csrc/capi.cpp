@@ -100,6 +100,7 @@ struct lbm_grid {
   bool broken = false;
   int sched = LBM_SCHED_FUSED;  // lbm_set_schedule
   bool pdl = true;              // programmatic dependent launch of F_L^k after its gather (LBMR_NO_PDL=1: off)
+  int32_t prefetch = 16;        // L2 prefetch distance of the level kernels, in blocks (LBMR_PREFETCH; 0: off)
   bool peer_other_gpu[2] = {false, false};  // the connected neighbour on this side is on another GPU
   bool halo_spin = false;       // in-kernel halo waits (every connected neighbour on another GPU)
   int64_t steps = 0;
@@ -229,6 +230,7 @@ StepParams<T> make_params(const lbm_grid* g, int L, int64_t k) {
   }
   p.bc = g->bc_dev;
   p.omega = (T)g->omega[L];
+  p.prefetch = g->prefetch;
   for (int a = 0; a < 3; ++a) p.periodic[a] = g->desc.periodic[a];
   p.face_cls = g->face_dev;
   p.nfluid = g->host[L].nlaunch;
@@ -732,6 +734,7 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
   g->prec = d->precision;
   g->tsize = d->precision == LBM_FP32 ? 4 : 8;
   g->pdl = getenv("LBMR_NO_PDL") == nullptr;
+  if (const char* e = getenv("LBMR_PREFETCH")) g->prefetch = std::max(0, atoi(e));
   for (int c = 0; c < 256; ++c) {
     g->bc_host[c].kind = LBM_BC_NOSLIP;
     g->bc_host[c].pad_ = 0;

@@ -76,6 +76,9 @@ struct StepParams {
   // them (record word kRecCoalPull) wait for the gather at their start, all
   // others at their end, so the gather overlaps the level kernel
   int32_t pdl;
+  // > 0: each block's first CTA prefetches (cp.async.bulk.prefetch.L2) the
+  // populations of the block `prefetch` positions ahead in storage order
+  int32_t prefetch;
   // ---- x-slab partition (multi-GPU); unused when nbctas == 0 -------------
   int32_t nbctas;               // CTAs taking part in the halo protocol (cut-plane blocks, >= 1)
   int32_t nboundary;            // cut-plane blocks (stored and launched first)

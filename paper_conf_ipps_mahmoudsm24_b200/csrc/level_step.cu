@@ -873,6 +873,25 @@ struct StepCta {
   static constexpr int min_blocks = (PlainOcc<Q, T, COLL>::value * 256) / threads;
 };
 
+// L2 prefetch (P.prefetch blocks ahead in storage order): the first CTA of a
+// block has one thread ask the TMA unit (cp.async.bulk.prefetch.L2, SASS
+// UBLKPF) to bring the populations of block blk + prefetch — contiguous, Q x
+// 512 values — into L2, so the CTAs that process that block shortly after
+// pull from L2 instead of DRAM.  The resident warps' registers bound the
+// loads in flight; the bulk prefetch adds memory-level parallelism without
+// registers.  Measured (16 blocks ahead): cfg5 fp32 +3 %, fp64 +3 % (finest
+// level 0.954 -> 0.978 of the copy peak), Tab. I s3 fp64 KBC +10 % (0.77 ->
+// 0.85), cfg4 KBC fp32 +8 % (0.72 -> 0.78); 512 blocks ahead thrashes L2.
+template <int Q, typename T>
+__device__ __forceinline__ void prefetch_block(const StepParams<T>& P, int blk) {
+  if (P.prefetch <= 0 || threadIdx.x != 0) return;
+  const int pb = blk + P.prefetch;
+  if (pb >= P.nfluid) return;
+  const T* a = P.src + (size_t)pb * (Q * kCells);
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a), "r"((unsigned)(Q * kCells * sizeof(T)))
+               : "memory");
+}
+
 // Programmatic dependent launch (sm_90+): wait until the preceding kernel of
 // the stream (the coalescence gather) has completed and its writes are
 // visible; let the following kernel launch early.
@@ -890,6 +909,7 @@ __global__ void __launch_bounds__(StepCta<Q, COLL, T>::threads, StepCta<Q, COLL,
     return;
   }
   const int b = (int)blockIdx.x;
+  if ((b % PB) == 0) prefetch_block<Q, T>(P, b / PB);
   // under PDL the gather may still be running: CTAs whose block pulls a
   // coalescence ghost wait for it first, the others after their work
   const bool early = P.pdl && __ldg(P.nbr + (b / PB) * kRec + kRecCoalPull) != 0;
@@ -963,6 +983,7 @@ __global__ void __launch_bounds__(kHaloCtaThreads, (PlainOcc<Q, T, COLL>::value 
   const bool fill = (int)blockIdx.x >= main;
   const bool proto = (int)blockIdx.x < P.nbctas || fill;
   if (P.halo_spin && proto) halo_spin_cta(P.flags, P.has_nb[0], P.has_nb[1]);
+  if (!fill && ((int)blockIdx.x % PB) == 0) prefetch_block<Q, T>(P, blk);
   if (fill) {
     trail_fill<Q, T>(P, ((int)blockIdx.x - main) * NT + threadIdx.x);
   } else if (blk < P.nfluid) {
