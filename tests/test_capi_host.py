@@ -181,3 +181,35 @@ def test_builder_statistics_of_the_baseline_configs():
     sc = [gi.special_cells[L] / gi.leaves[L] for L in range(4)]
     assert sc[0] < 0.090 and sc[1] < 0.065 and sc[3] < 0.01
     assert gi.special_cells[2] == 0
+
+
+# ---------------------------------------------------------------- block-grid alignment
+def _offset_problem():
+    """2 levels, the refined box starting at coarse x = 3 (level-1 x = 6, 6 mod 8 = 6):
+    the builder should shift level 1's block grid by 2 in x."""
+    n = (16, 12, 10)
+    masks = I._box_masks(n, [((3, 11), (2, 8), (0, 10))])
+    return I.Problem(name="offset", nx=n[0], ny=n[1], nz=n[2], masks=masks, face_bc=(2,) * 6, Q=19,
+                     omega0=1.2, bc={2: (I.BC_NOSLIP, (0.0, 0.0, 0.0))})
+
+
+def test_block_grid_offsets_align_level_faces(monkeypatch):
+    p = _offset_problem()
+    a = lbmr.analyze_problem(p)
+    off = [[a.block_offset[L][k] for k in range(3)] for L in range(p.levels)]
+    # level 1 fluid region x in [6, 22): faces at 6 and 22 (both 6 mod 8) -> offset 2;
+    # y in [4, 16): faces 4 and 16 (4 and 0 mod 8) and the domain faces 0 and 24 -> 0 wins
+    assert off[1][0] == 2, off
+    assert off[0] == [0, 0, 0], off
+    monkeypatch.setenv("LBMR_NO_BLOCK_ALIGN", "1")
+    b = lbmr.analyze_problem(p)
+    assert [[b.block_offset[L][k] for k in range(3)] for L in range(2)] == [[0, 0, 0], [0, 0, 0]]
+    # same leaves and work (the aligned grid stores its explosion ghosts in ghost-only blocks
+    # outside the fluid region's rows, so it may hold more population blocks)
+    assert list(a.leaves[:2]) == list(b.leaves[:2])
+
+
+def test_block_grid_offsets_zero_on_periodic_axes():
+    p = I.random_balanced(31, n=(12, 10, 9), levels=3, p_refine=0.6, periodic=(1, 1, 1), p_bc=0.0)
+    a = lbmr.analyze_problem(p)
+    assert all(a.block_offset[L][k] == 0 for L in range(3) for k in range(3))

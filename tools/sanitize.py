@@ -1,9 +1,15 @@
 """Short runs for compute-sanitizer (T15): cfg1 cavity (2 levels), a random
-2:1 grid with BC leaves, and a 2-slab partition, fp32 and fp64."""
-import os, sys
+2:1 grid with BC leaves, the KBC cavity, every fusion-ablation schedule of
+the paper (Fig. 4b-4f: split E / A / O kernels, the atomic scatter
+Accumulate) on the reduced tunnel, and 2-slab partitions with the
+one-thread wait kernels and with the in-kernel waits, fp32 and fp64."""
+import os
+import sys
+
 sys.path.insert(0, os.getcwd())
-import lbm_inputs as I
-from paper_conf_ipps_mahmoudsm24_b200 import lbmr
+import lbm_inputs as I  # noqa: E402
+from paper_conf_ipps_mahmoudsm24_b200 import lbmr  # noqa: E402
+
 for prec in (lbmr.FP32, lbmr.FP64):
     for prob in (I.cavity2("r"), I.random_balanced(33, n=(9, 11, 10), levels=4, p_refine=0.5),
                  I.cavity4_kbc("mini")):
@@ -12,8 +18,18 @@ for prec in (lbmr.FP32, lbmr.FP64):
         g.macroscopic(prob.levels - 1)
         g.stats()
         g.close()
-    pg = lbmr.PartitionedGrid(I.cavity2("r"), 2, precision=prec)
-    pg.step(2)
-    pg.macroscopic(1)
-    pg.close()
+    prob = I.tunnel4(scale=5)
+    for fig, mode in lbmr.FIG4.items():
+        g = lbmr.grid_from_problem(prob, precision=prec)
+        g.set_schedule(mode)
+        g.step(2)
+        g.stats()
+        g.close()
+    for spin in ("0", "1"):
+        os.environ["LBMR_HALO_SPIN"] = spin
+        pg = lbmr.PartitionedGrid(I.cavity2("r"), 2, precision=prec)
+        pg.step(2)
+        pg.macroscopic(1)
+        pg.close()
+    os.environ.pop("LBMR_HALO_SPIN", None)
 print("sanitize run done")
