@@ -283,11 +283,19 @@ bool level_has_coal(const lbm_grid* g, int L) {
   return L >= 0 && L + 1 < g->levels && !g->host[L].coal_fill.empty();
 }
 
-void launch_gather(lbm_grid* g, int L, const void* fa, const void* fb, void* dst, int mode) {
+// Programmatic dependent launch of every kernel of the product schedule
+// after the previous one (single rank, or ranks whose halo waits are
+// in-kernel): a kernel's CTAs become resident during the previous kernel's
+// tail instead of after its completion (LBMR_NO_PDL=1: off).
+bool pdl_chain(const lbm_grid* g) {
+  return g->pdl && !(g->sched & (LBM_SCHED_UNFUSED | kAblationBits)) && (g->n_ranks == 1 || g->halo_spin);
+}
+
+void launch_gather(lbm_grid* g, int L, const void* fa, const void* fb, void* dst, int mode, bool chain = false) {
   const HostLevel& H = g->host[L];
   const bool spin = g->n_ranks > 1 && g->halo_spin;
   launch_coalesce(g->Q, g->prec, fa, fb, dst, g->dev[L].coal_fill, g->dev[L].coal_cand, H.coal_n[0], H.coal_n[1], mode,
-                  g->stream, spin ? g->flags : nullptr, g->has_nb[0], g->has_nb[1]);
+                  g->stream, spin ? g->flags : nullptr, g->has_nb[0], g->has_nb[1], chain ? 1 : 0);
 }
 
 // In-kernel halo waits when every connected neighbour is on another GPU
@@ -370,7 +378,7 @@ void launch_F_typed(lbm_grid* g, int L, int64_t k, int kind, cudaEvent_t mid = n
     void* dst = g->dev[L].pop[k & 1];
     if (!(sched & (LBM_SCHED_SPLIT_A | LBM_SCHED_ATOMIC_A))) {
       launch_gather(g, L, g->dev[L + 1].pop[1], g->dev[L + 1].pop[0], dst,
-                    (sched & LBM_SCHED_SPLIT_O) ? 0 : kCoalDivide);
+                    (sched & LBM_SCHED_SPLIT_O) ? 0 : kCoalDivide, pdl_chain(g) && !mid_stamp);
       // the product schedule: F_L^k is the programmatic dependent of the
       // gather (its CTAs that do not pull coalescence ghosts overlap it)
       p.pdl = (g->n_ranks == 1 && !(sched & (LBM_SCHED_UNFUSED | kAblationBits)) && g->pdl) ? 1 : 0;
@@ -382,6 +390,9 @@ void launch_F_typed(lbm_grid* g, int L, int64_t k, int kind, cudaEvent_t mid = n
   ablation_params<T>(g, L, k, p);
   if (mid) cudaEventRecord(mid, g->stream);
   if (mid_stamp) launch_stamp(mid_stamp, 0, g->stream);
+  // the level kernel follows the previous kernel programmatically, unless a
+  // halo wait kernel (ranks sharing a GPU) or a profiling stamp sits between
+  p.pdl_chain = (pdl_chain(g) && !mid_stamp && !mid) ? 1 : 0;
   if (sched & LBM_SCHED_UNFUSED) {  // S_L^k then C_L^{k+1} in place (fusion ablation)
     StepParams<T> sp = p;  // the stream half: no scatter (nothing collided yet)
     sp.sc_qoff = nullptr;

@@ -76,6 +76,9 @@ struct StepParams {
   // them (record word kRecCoalPull) wait for the gather at their start, all
   // others at their end, so the gather overlaps the level kernel
   int32_t pdl;
+  // 1: launched as the programmatic dependent of the previous kernel of the
+  // step (PDL chain): CTAs wait for it at their start, then trigger the next
+  int32_t pdl_chain;
   // > 0: each block's first CTA prefetches (cp.async.bulk.prefetch.L2) the
   // populations of the block `prefetch` positions ahead in storage order
   int32_t prefetch;
@@ -104,9 +107,12 @@ struct StepParams {
 enum { kCoalFromDst = 1, kCoalDivide = 2 };
 // spin_flags (partitioned grid whose neighbours are on other GPUs): every CTA
 // first waits in-kernel for the neighbours' previous kernels (halo protocol).
+// pdl_chain: launched as the programmatic dependent of the previous level
+// kernel (it waits for it at entry).
 void launch_coalesce(int Q, int precision, const void* fa, const void* fb, void* dst, const uint32_t* fill,
                      const uint32_t* cand, int64_t n_main, int64_t n_ovf, int mode, cudaStream_t s,
-                     const unsigned long long* spin_flags = nullptr, int nb0 = 0, int nb1 = 0);
+                     const unsigned long long* spin_flags = nullptr, int nb0 = 0, int nb1 = 0,
+                     int pdl_chain = 0);
 
 // rho / u (double) of n cells given by population cell index block*512+local
 // (-1 -> NaN), read from the post-collision buffer `pop`.

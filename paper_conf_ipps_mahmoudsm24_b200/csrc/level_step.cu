@@ -903,7 +903,15 @@ __global__ void __launch_bounds__(StepCta<Q, COLL, T>::threads, StepCta<Q, COLL,
     level_step_all(const StepParams<T> P) {
   constexpr int NT = StepCta<Q, COLL, T>::threads, PB = StepCta<Q, COLL, T>::per_block;
   const int main = P.nfluid * PB;
+  // PDL chain (P.pdl_chain): launched as the programmatic dependent of the
+  // previous level kernel, so this grid's CTAs become resident during that
+  // kernel's tail; they wait for its completion before touching memory and
+  // then let the next kernel launch.  After the coalescence gather (P.pdl)
+  // only the CTAs that pull its ghosts wait first, the others after their
+  // work; either way the kernel completes only after its predecessor.
+  if (P.pdl_chain && !P.pdl) pdl_wait();
   if ((int)blockIdx.x >= main) {  // trailing CTAs refresh the explosion ghosts
+    if (P.pdl || P.pdl_chain) pdl_launch_dependents();
     trail_fill<Q, T>(P, ((int)blockIdx.x - main) * NT + threadIdx.x);
     if (P.pdl) pdl_wait();  // this kernel completes only after the gather
     return;
@@ -914,6 +922,7 @@ __global__ void __launch_bounds__(StepCta<Q, COLL, T>::threads, StepCta<Q, COLL,
   // coalescence ghost wait for it first, the others after their work
   const bool early = P.pdl && __ldg(P.nbr + (b / PB) * kRec + kRecCoalPull) != 0;
   if (early) pdl_wait();
+  if (P.pdl || P.pdl_chain) pdl_launch_dependents();
   step_cell<Q, COLL, T, false, true, NT>(P, b / PB, (b % PB) * NT + threadIdx.x);
   if (P.sc_qoff) accumulate_scatter<T, NT>(P, b / PB, (b % PB) * NT);
   if (P.pdl && !early) pdl_wait();
@@ -982,6 +991,10 @@ __global__ void __launch_bounds__(kHaloCtaThreads, (PlainOcc<Q, T, COLL>::value 
   // read L-1 halo cells) count towards this kernel's completion signal
   const bool fill = (int)blockIdx.x >= main;
   const bool proto = (int)blockIdx.x < P.nbctas || fill;
+  if (P.pdl_chain) {  // PDL chain: resident during the previous kernel's tail (see level_step_all)
+    pdl_wait();
+    pdl_launch_dependents();
+  }
   if (P.halo_spin && proto) halo_spin_cta(P.flags, P.has_nb[0], P.has_nb[1]);
   if (!fill && ((int)blockIdx.x % PB) == 0) prefetch_block<Q, T>(P, blk);
   if (fill) {
@@ -1173,8 +1186,9 @@ __global__ void __launch_bounds__(256) coalesce_kernel(const T* __restrict__ fa,
                                                        const uint32_t* __restrict__ fill,
                                                        const uint32_t* __restrict__ cand, int64_t nmain, int64_t novf,
                                                        int mode, const unsigned long long* spin_flags, int nb0,
-                                                       int nb1) {
-  pdl_launch_dependents();  // the level kernel after it may start (it waits where it needs us)
+                                                       int nb1, int pdl_chain) {
+  if (pdl_chain) pdl_wait();  // launched as the PDL dependent of the previous level kernel
+  pdl_launch_dependents();    // the level kernel after it may start (it waits where it needs us)
   // partitioned grid on distinct GPUs: the candidates may be halo cells of the
   // finer level, written by the neighbour's last fine kernel
   if (spin_flags) halo_spin_cta(spin_flags, nb0, nb1);
@@ -1247,19 +1261,42 @@ void launch_halo_wait(const unsigned long long* flags, int nb0, int nb1, cudaStr
   halo_wait_kernel<<<1, 1, 0, s>>>(flags, nb0, nb1);
 }
 
+// cudaLaunchKernelEx with the programmatic-stream-serialization attribute
+// (pdl = 1) or a plain launch
+template <typename Kern, typename... Args>
+static void launch_maybe_pdl(bool pdl, Kern kernel, dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                             Args... args) {
+  if (!pdl) {
+    kernel<<<grid, block, smem, s>>>(args...);
+    return;
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  cudaLaunchKernelEx(&cfg, kernel, args...);
+}
+
 void launch_coalesce(int Q, int precision, const void* fa, const void* fb, void* dst, const uint32_t* fill,
                      const uint32_t* cand, int64_t n_main, int64_t n_ovf, int mode, cudaStream_t s,
-                     const unsigned long long* spin_flags, int nb0, int nb1) {
+                     const unsigned long long* spin_flags, int nb0, int nb1, int pdl_chain) {
   (void)Q;
   const int64_t n = n_main + n_ovf;
   if (n <= 0) return;
   const unsigned grid = (unsigned)((n + 255) / 256);
   if (precision == LBM_FP32)
-    coalesce_kernel<float><<<grid, 256, 0, s>>>((const float*)fa, (const float*)fb, (float*)dst, fill, cand, n_main,
-                                                 n_ovf, mode, spin_flags, nb0, nb1);
+    launch_maybe_pdl(pdl_chain != 0, coalesce_kernel<float>, dim3(grid), dim3(256), 0, s, (const float*)fa,
+                     (const float*)fb, (float*)dst, fill, cand, n_main, n_ovf, mode, spin_flags, nb0, nb1, pdl_chain);
   else
-    coalesce_kernel<double><<<grid, 256, 0, s>>>((const double*)fa, (const double*)fb, (double*)dst, fill, cand,
-                                                  n_main, n_ovf, mode, spin_flags, nb0, nb1);
+    launch_maybe_pdl(pdl_chain != 0, coalesce_kernel<double>, dim3(grid), dim3(256), 0, s, (const double*)fa,
+                     (const double*)fb, (double*)dst, fill, cand, n_main, n_ovf, mode, spin_flags, nb0, nb1,
+                     pdl_chain);
 }
 
 // ---------------------------------------------------------------- dispatch
@@ -1283,7 +1320,7 @@ static void launch_typed(int kind, const void* params, cudaStream_t s) {
     dim3 grid(kHaloCtasPerBlock * std::max(p.nfluid, 1) + halo_fill_ctas(trail_count(p)));
     const size_t hs = (size_t)Q * kHaloCtaThreads * sizeof(T);
     if (kind == 1) level_step_halo<Q, COLL, T, false><<<grid, dim3(kHaloCtaThreads), 0, s>>>(p);
-    else level_step_halo<Q, COLL, T, true><<<grid, dim3(kHaloCtaThreads), hs, s>>>(p);
+    else launch_maybe_pdl(p.pdl_chain != 0, level_step_halo<Q, COLL, T, true>, grid, dim3(kHaloCtaThreads), hs, s, p);
     return;
   }
   if (p.nfluid <= 0 && trail_count(p) <= 0) return;
@@ -1298,21 +1335,7 @@ static void launch_typed(int kind, const void* params, cudaStream_t s) {
     const int gct = (trail_count(p) + NT - 1) / NT;
     const dim3 grid(p.nfluid * StepCta<Q, COLL, T>::per_block + gct), blk(NT);
     const size_t smem = (size_t)Q * NT * sizeof(T);
-    if (p.pdl) {
-      cudaLaunchConfig_t cfg = {};
-      cfg.gridDim = grid;
-      cfg.blockDim = blk;
-      cfg.dynamicSmemBytes = smem;
-      cfg.stream = s;
-      cudaLaunchAttribute attr[1];
-      attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-      attr[0].val.programmaticStreamSerializationAllowed = 1;
-      cfg.attrs = attr;
-      cfg.numAttrs = 1;
-      cudaLaunchKernelEx(&cfg, level_step_all<Q, COLL, T>, p);
-    } else {
-      level_step_all<Q, COLL, T><<<grid, blk, smem, s>>>(p);
-    }
+    launch_maybe_pdl(p.pdl || p.pdl_chain, level_step_all<Q, COLL, T>, grid, blk, smem, s, p);
   }
 }
 
