@@ -34,6 +34,10 @@
 
 namespace lbmr {
 
+// griddepcontrol.wait (sm_90+): block until the stream's preceding kernel
+// (programmatic dependent launch) has completed and its writes are visible
+__device__ __forceinline__ void griddep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
 __constant__ int c_ex[27] = {LBMR_EX_LIST};
 __constant__ int c_ey[27] = {LBMR_EY_LIST};
 __constant__ int c_ez[27] = {LBMR_EZ_LIST};
@@ -674,8 +678,11 @@ __device__ __forceinline__ void accumulate_scatter(const StepParams<T>& P, int b
 
 // Minimum resident CTAs per SM (register budget 65536 / (256 * MINB)),
 // chosen per variant from ptxas -v and measurement.
+// D3Q19 fp32: 5 units = 48 registers (round 2, with the L2 prefetch and the
+// in-record PDL gate: cfg5 +1.4 %, cfg3 +1.9 %, uniform512 +1.1 % over 6
+// units = 40 registers; round 1 without the prefetch measured 6 better)
 #ifndef LBMR_OCC_Q19F
-#define LBMR_OCC_Q19F 6
+#define LBMR_OCC_Q19F 5
 #endif
 #ifndef LBMR_OCC_KBCF
 #define LBMR_OCC_KBCF 4
@@ -759,13 +766,17 @@ template <int Q>
 constexpr bool kEarlyBounce = (Q == 27);
 
 template <int Q, int COLL, typename T, bool HALO, bool COLLIDE = true, int NT = 256>
-__device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t) {
+__device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t, bool pdl_gate = false) {
   constexpr unsigned FULL = 0xffffffffu;
   const int lane = threadIdx.x & 31;
   const int* R = P.nbr + blk * kRec;
   const int rec = __ldg(R + lane);
   const uint32_t fm = (uint32_t)__ldg(R + kRecFluid + (t >> 5));
   const uint32_t sm = (uint32_t)__ldg(R + kRecSpecial + (t >> 5));
+  // PDL after the coalescence gather: a warp whose block pulls coalescence
+  // ghosts waits for the gather before its pulls (the flag rides in the
+  // record the warp has just loaded: no extra round trip)
+  if (pdl_gate && __shfl_sync(FULL, rec, kRecCoalPull) != 0) griddep_wait();
   const PullGeom G(t);
   T g[Q];
   const unsigned own = (unsigned)blk * (unsigned)(Q * kCells) + (unsigned)t;
@@ -895,7 +906,7 @@ __device__ __forceinline__ void prefetch_block(const StepParams<T>& P, int blk) 
 // Programmatic dependent launch (sm_90+): wait until the preceding kernel of
 // the stream (the coalescence gather) has completed and its writes are
 // visible; let the following kernel launch early.
-__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_wait() { griddep_wait(); }
 __device__ __forceinline__ void pdl_launch_dependents() { asm volatile("griddepcontrol.launch_dependents;" :::); }
 
 template <int Q, int COLL, typename T>
@@ -918,14 +929,13 @@ __global__ void __launch_bounds__(StepCta<Q, COLL, T>::threads, StepCta<Q, COLL,
   }
   const int b = (int)blockIdx.x;
   if ((b % PB) == 0) prefetch_block<Q, T>(P, b / PB);
-  // under PDL the gather may still be running: CTAs whose block pulls a
-  // coalescence ghost wait for it first, the others after their work
-  const bool early = P.pdl && __ldg(P.nbr + (b / PB) * kRec + kRecCoalPull) != 0;
-  if (early) pdl_wait();
   if (P.pdl || P.pdl_chain) pdl_launch_dependents();
-  step_cell<Q, COLL, T, false, true, NT>(P, b / PB, (b % PB) * NT + threadIdx.x);
+  // under PDL the gather may still be running: warps whose block pulls a
+  // coalescence ghost wait for it before their pulls (inside step_cell), all
+  // others after their work (a second wait returns at once)
+  step_cell<Q, COLL, T, false, true, NT>(P, b / PB, (b % PB) * NT + threadIdx.x, P.pdl != 0);
   if (P.sc_qoff) accumulate_scatter<T, NT>(P, b / PB, (b % PB) * NT);
-  if (P.pdl && !early) pdl_wait();
+  if (P.pdl) pdl_wait();
 }
 
 // Partitioned variant: grid = 4 * max(nfluid, 1) quarter-block CTAs; the first nbctas run
