@@ -762,8 +762,11 @@ __device__ __forceinline__ void halo_store(const StepParams<T>& P, const T (&g)[
 // Bounce copies issued with the pulls (per-warp union masks, lattice.h
 // kBounceWords) or after the cell's info: measured per lattice — D3Q27
 // (cfg4: every warp walls) +3 % BGK, +20 % KBC; D3Q19 (cfg5) -0.4 %.
+#ifndef LBMR_EARLY_BOUNCE_Q19
+#define LBMR_EARLY_BOUNCE_Q19 0
+#endif
 template <int Q>
-constexpr bool kEarlyBounce = (Q == 27);
+constexpr bool kEarlyBounce = (Q == 27) || LBMR_EARLY_BOUNCE_Q19;
 
 template <int Q, int COLL, typename T, bool HALO, bool COLLIDE = true, int NT = 256>
 __device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t, bool pdl_gate = false) {
