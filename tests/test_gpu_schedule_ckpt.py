@@ -231,3 +231,21 @@ def test_set_bc_mid_run_applies_from_next_step(prec):
     _same(changed, _fields(k, prob.levels))
     k.close()
     assert not np.array_equal(np.nan_to_num(changed[0][1]), np.nan_to_num(unchanged[0][1]))
+
+
+@pytest.mark.parametrize("env", [{"LBMR_NO_PDL": "1"}, {"LBMR_PREFETCH": "0"}, {"LBMR_PREFETCH": "200"},
+                                 {"LBMR_NO_BLOCK_ALIGN": "1"}, {"LBMR_BLOCK_ORDER": "hilbert"}],
+                         ids=["no_pdl", "no_prefetch", "far_prefetch", "no_align", "hilbert"])
+def test_performance_switches_do_not_change_results(env, monkeypatch):
+    """The programmatic-dependent-launch chain, the L2 prefetch distance, the
+    block-grid alignment and the block order are performance choices only:
+    bitwise the same fields (fp64 and fp32) with each switched."""
+    for prec in (FP64, FP32):
+        for name in ("tunnel_s5", "kbc_mini"):
+            prob = PROBLEMS[name]()
+            ref = _run(prob, prec, 3, _lbmr().SCHED_FUSED)
+            with monkeypatch.context() as m:
+                for k, v in env.items():
+                    m.setenv(k, v)
+                got = _run(prob, prec, 3, _lbmr().SCHED_FUSED)
+            _same(ref, got)
