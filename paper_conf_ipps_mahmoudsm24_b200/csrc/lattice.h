@@ -79,6 +79,10 @@ constexpr unsigned kNoBCSource = 0xffffffffu;
 //  kLinkTemp   w0 = index into the level's volumetric averages
 constexpr unsigned kLinkSame = 0, kLinkCoarse = 1, kLinkBC = 2, kLinkFace = 3, kLinkCoal = 4, kLinkTemp = 5;
 
+// explosion-ghost fill entry {ghost cell, parent cell, mask}: bit 31 of the
+// mask = the ghost is the only live cell of its 8-cell x-row (whole-row store)
+constexpr unsigned kGhostRowOwn = 1u << 31;
+
 // volumetric-variant expression tags (which buffer the population index is in)
 //  fill list of level L (run by F_L^{k-1}):  kVtA = C_L^{k-1}, kVtB = C_{L-1}
 //  average list of level L (before F_L^k):   kVtA = C_L^k, kVtB = C_{L+1}^{2k-1}, kVtC = C_{L+1}^{2k}

@@ -592,6 +592,24 @@ __device__ __forceinline__ void ghost_fill_one(const StepParams<T>& P, int i) {
   const uint32_t mask = __ldg(P.ghost_fill + 3 * i + 2);
   T* d = P.dst + (gc >> 9) * (unsigned)(Q * kCells) + (gc & 511u);
   const T* s = P.gsrc + (pc >> 9) * (unsigned)(Q * kCells) + (pc & 511u);
+  if (mask & kGhostRowOwn) {
+    // the ghost is the row's only live cell: store the value over the whole
+    // 8-cell row (aligned full sectors; the other seven cells are never read)
+    T* r = d - (gc & 7u);
+#pragma unroll
+    for (int q = 1; q < Q; ++q)
+      if ((mask >> q) & 1u) {
+        const T v = __ldg(s + q * kCells);
+        if constexpr (sizeof(T) == 4) {
+          float4* w = reinterpret_cast<float4*>(r + q * kCells);
+          w[0] = w[1] = make_float4(v, v, v, v);
+        } else {
+          double2* w = reinterpret_cast<double2*>(r + q * kCells);
+          w[0] = w[1] = w[2] = w[3] = make_double2(v, v);
+        }
+      }
+    return;
+  }
 #pragma unroll
   for (int q = 1; q < Q; ++q)
     if ((mask >> q) & 1u) d[q * kCells] = __ldg(s + q * kCells);
