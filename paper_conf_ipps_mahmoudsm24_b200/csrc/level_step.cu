@@ -453,15 +453,20 @@ struct PullGeom {
   }
 };
 
-// Streaming loads / stores of populations (variants selected at build time,
-// measured in tools/gpu_variants.sh): LBMR_LDVAR 0 = ld.global.nc, 1 = +
-// L2::256B prefetch, 2 = + L1::no_allocate + L2::256B, 3 = L1::no_allocate;
-// LBMR_STVAR 0 = st.global, 1 = st.global.cs (evict-first).
+// Streaming loads / stores of populations (variants selected at build time):
+// LBMR_LDVAR 0 = ld.global.nc, 1 = + L2::256B prefetch, 2 = + L1::no_allocate
+// + L2::256B, 3 = L1::no_allocate; LBMR_STVAR 0 = st.global, 1 = st.global.cs
+// (evict-first).  Re-measured with the L2 bulk prefetch (round 2, 3 runs):
+// 0 / 1 beats the round-1 choice 1 / 0 by 1.0 % on cfg5 fp32 (finest level
+// 0.963 -> 0.973), 0.9 % on cfg5 fp64, 0.5 % on Tab. I s3 fp64 (cfg4 KBC
+// equal): the bulk prefetch replaces the per-load 256-byte L2 prefetch hint,
+// and evict-first stores leave L2 to the neighbour blocks' halo reads;
+// no_allocate in L1 loses the in-CTA reuse of neighbour rows (-15 %).
 #ifndef LBMR_LDVAR
-#define LBMR_LDVAR 1
+#define LBMR_LDVAR 0
 #endif
 #ifndef LBMR_STVAR
-#define LBMR_STVAR 0
+#define LBMR_STVAR 1
 #endif
 template <typename T>
 __device__ __forceinline__ T ld_pop(const T* p) {
