@@ -52,7 +52,8 @@ PAPER_MLUPS = {f"sphere_tab1_s{_s}": I.TAB1[_s]["ours_mlups"] for _s in (1, 2, 3
 # lbm_set_schedule bit sets (lbmr.h): the product, the C/S split, the graph-free
 # launch path, and the paper's Fig. 4 fusion configurations (lbmr.FIG4)
 SCHEDULES = {"fused": 0, "unfused": 1, "nograph": 2, "unfused_nograph": 3,
-             "fig4b": 1 | 4 | 8 | 32, "fig4c": 1 | 4 | 16 | 32, "fig4d": 1 | 8 | 32, "fig4e": 1 | 16, "fig4f": 16}
+             "fig4b": 1 | 4 | 8 | 32, "fig4c": 1 | 4 | 16 | 32, "fig4d": 1 | 8 | 32, "fig4e": 1 | 16, "fig4f": 16,
+             "cta_gather": 64}  # A+A+O gathered inside F_L^k by each CTA (no gather kernel)
 N_PROBE = 4096  # e2e monitoring cells
 # bounded oracle sample for --impl reference (one coarse step per timed step)
 REF_SAMPLE = {

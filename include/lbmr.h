@@ -91,11 +91,15 @@ typedef struct {
   int64_t total_blocks[16];          /* all stored blocks incl. refined/BC-only                   */
   int64_t device_bytes;              /* device memory held by the grid                            */
   int64_t steps_done;                /* coarse steps since the last init                          */
-  int64_t launches_per_step;         /* every kernel of one fused coarse step: the level steps plus
-                                        one coalescence gather before each F_L^k whose level has
-                                        coalescence ghosts                                          */
+  int64_t launches_per_step;         /* every kernel of one coarse step under the current schedule:
+                                        the level steps (the product gathers coalescence inside
+                                        them), plus the separate gather / split kernels and halo
+                                        waits other schedules add                                   */
   int32_t block_offset[16][3];       /* per level and axis: level cell c lies in 8^3 block
                                         (c + off) >> 3 (builder-chosen alignment)     */
+  int64_t coal_links[16];            /* per level: coalescence links with B != {} (Eq.11 gathers
+                                        per F_L^k)                                                  */
+  int64_t coal_wide[16];             /* of those, links with |B| > 4 (concave interface edges)      */
 } lbm_grid_info;
 
 /* Build the block-sparse multi-level grid (§V) from per-level masks.
@@ -178,8 +182,10 @@ lbm_status lbm_profile_levels(lbm_grid* g, int32_t n_coarse, double* ms_per_leve
  * accumulated values), §IV and Fig. 4.
  *  LBM_SCHED_FUSED     (0) one fused kernel F_L^k per level-substep (S + E +
  *                      O + BC + C), 2Q values moved per leaf, and one small
- *                      gather kernel before it doing A + A + O from the two
- *                      retained fine buffers (deterministic) — the product.
+ *                      warp-cooperative gather kernel before it doing A + A +
+ *                      O from the two retained fine buffers (deterministic,
+ *                      warp shuffles; F_L^k its programmatic dependent) — the
+ *                      product.
  *  LBM_SCHED_UNFUSED   (1) C and S separate: a stream-only kernel S_L^k then
  *                      an in-place collision C_L^{k+1} (4Q values per leaf).
  *  LBM_SCHED_NO_GRAPH  (2) launch the kernels one by one instead of replaying
@@ -197,6 +203,11 @@ lbm_status lbm_profile_levels(lbm_grid* g, int32_t n_coarse, double* ms_per_leve
  *  LBM_SCHED_SPLIT_O   (32) O's division by 2|B| as its own kernel before
  *                      the coarse S / F (otherwise fused into the last
  *                      Accumulate, or pre-scaled atomic terms).
+ *  LBM_SCHED_CTA_GATHER (64) A + A + O inside F_L^k instead of the gather
+ *                      kernel: each CTA first gathers its own cells'
+ *                      coalescence links (warp shuffles, into its shared
+ *                      staging column); ignored with UNFUSED, SPLIT_A,
+ *                      ATOMIC_A or SPLIT_O (which need the ghost slots).
  * The paper's configurations: Fig. 4b modified baseline = UNFUSED | SPLIT_E |
  * SPLIT_A | SPLIT_O; 4c = UNFUSED | SPLIT_E | ATOMIC_A | SPLIT_O; 4d (SE
  * fused) = UNFUSED | SPLIT_A | SPLIT_O; 4e (CA, SE, SO fused) = UNFUSED |
@@ -212,7 +223,8 @@ enum {
   LBM_SCHED_SPLIT_E = 4,
   LBM_SCHED_SPLIT_A = 8,
   LBM_SCHED_ATOMIC_A = 16,
-  LBM_SCHED_SPLIT_O = 32
+  LBM_SCHED_SPLIT_O = 32,
+  LBM_SCHED_CTA_GATHER = 64
 };
 lbm_status lbm_set_schedule(lbm_grid* g, int32_t mode);
 

@@ -63,6 +63,11 @@ struct DevLevel {
   uint32_t* ghost_fill = nullptr;
   uint32_t* coal_fill = nullptr;
   uint32_t* coal_cand = nullptr;
+  uint32_t* coal_wcand = nullptr;  // warp-cooperative gather units
+  uint32_t* coal_wdst = nullptr;
+  uint32_t* cg_qoff = nullptr;    // coalescence fused into the level kernel (product schedule)
+  uint32_t* cg_cand = nullptr;
+  uint32_t* cg_dest = nullptr;
   uint32_t* sc_qoff = nullptr;    // atomic Accumulate (ablation) scatter lists
   uint32_t* sc_items = nullptr;
   uint32_t* vfill = nullptr;   // volumetric variant lists (grid_builder.h)
@@ -100,9 +105,11 @@ struct lbm_grid {
   bool broken = false;
   int sched = LBM_SCHED_FUSED;  // lbm_set_schedule
   bool pdl = true;              // programmatic dependent launch of F_L^k after its gather (LBMR_NO_PDL=1: off)
+  bool gather_warp = false;      // warp-cooperative gather kernel (LBMR_GATHER_WARP=1; default thread per entry)
   int32_t prefetch = 16;        // L2 prefetch distance of the level kernels, in blocks (LBMR_PREFETCH; 0: off)
   bool peer_other_gpu[2] = {false, false};  // the connected neighbour on this side is on another GPU
   bool halo_spin = false;       // in-kernel halo waits (every connected neighbour on another GPU)
+  bool nb_other_gpu = false;    // every connected neighbour is on another GPU (halo_spin without the env override)
   int64_t steps = 0;
   int64_t device_bytes = 0;
   std::vector<void*> allocs;
@@ -275,9 +282,20 @@ StepParams<T> make_params(const lbm_grid* g, int L, int64_t k) {
 //   SPLIT_O    Coalescence's division by 2|B| as its own kernel O_L^k before
 //              the coarse S/F (otherwise fused: into the last gather, or
 //              pre-scaled atomic terms)
-// The product schedule (0) gathers A + A + O in one small kernel right before
-// F_L^k from the two retained fine buffers (deterministic, no atomics).
-constexpr int kAblationBits = LBM_SCHED_SPLIT_E | LBM_SCHED_SPLIT_A | LBM_SCHED_ATOMIC_A | LBM_SCHED_SPLIT_O;
+//   CTA_GATHER A + A + O inside F_L^k: each CTA gathers its own cells'
+//              coalescence links (no gather kernel)
+// The product schedule (0) gathers A + A + O in one small warp-cooperative
+// kernel right before F_L^k from the two retained fine buffers
+// (deterministic, no atomics), F_L^k its programmatic dependent.
+constexpr int kAblationBits =
+    LBM_SCHED_SPLIT_E | LBM_SCHED_SPLIT_A | LBM_SCHED_ATOMIC_A | LBM_SCHED_SPLIT_O | LBM_SCHED_CTA_GATHER;
+
+// Coalescence inside F_L^k (CTA_GATHER): not with the unfused S kernel
+// (256-thread CTAs), the split / atomic Accumulate or separate O.
+bool fused_gather(int sched) {
+  return (sched & LBM_SCHED_CTA_GATHER) &&
+         !(sched & (LBM_SCHED_UNFUSED | LBM_SCHED_SPLIT_A | LBM_SCHED_ATOMIC_A | LBM_SCHED_SPLIT_O));
+}
 
 bool level_has_coal(const lbm_grid* g, int L) {
   return L >= 0 && L + 1 < g->levels && !g->host[L].coal_fill.empty();
@@ -286,14 +304,32 @@ bool level_has_coal(const lbm_grid* g, int L) {
 // Programmatic dependent launch of every kernel of the product schedule
 // after the previous one (single rank, or ranks whose halo waits are
 // in-kernel): a kernel's CTAs become resident during the previous kernel's
-// tail instead of after its completion (LBMR_NO_PDL=1: off).
+// tail instead of after its completion (LBMR_NO_PDL=1: off).  Not when a
+// neighbour shares the GPU (in-kernel waits forced by LBMR_HALO_SPIN=1): the
+// dependent grid's parked CTAs could then hold the SM slots the neighbour's
+// kernel needs while our protocol CTAs spin for it.  On its own GPU a rank
+// cannot starve itself: the dependent grid launches only once every CTA of
+// the running kernel has started.
 bool pdl_chain(const lbm_grid* g) {
-  return g->pdl && !(g->sched & (LBM_SCHED_UNFUSED | kAblationBits)) && (g->n_ranks == 1 || g->halo_spin);
+  return g->pdl && !(g->sched & (LBM_SCHED_UNFUSED | (kAblationBits & ~LBM_SCHED_CTA_GATHER))) &&
+         (g->n_ranks == 1 || (g->halo_spin && g->nb_other_gpu));
 }
+
+// The gather kernel reads L+1 halo cells of a partitioned grid: every CTA
+// waits in-kernel when the neighbours are on other GPUs; otherwise a wait
+// kernel precedes it (with in-kernel waits forced on a shared GPU, spinning
+// gather CTAs could fill the SMs the neighbour's kernel needs).
+bool gather_spins(const lbm_grid* g) { return g->n_ranks > 1 && g->halo_spin && g->nb_other_gpu; }
 
 void launch_gather(lbm_grid* g, int L, const void* fa, const void* fb, void* dst, int mode, bool chain = false) {
   const HostLevel& H = g->host[L];
-  const bool spin = g->n_ranks > 1 && g->halo_spin;
+  const bool spin = gather_spins(g);
+  if (g->gather_warp) {
+    launch_coalesce_warp(g->prec, fa, fb, dst, g->dev[L].coal_wcand, g->dev[L].coal_wdst,
+                         (int64_t)H.coal_wdst.size(), H.coal_wpair, mode, g->stream, spin ? g->flags : nullptr,
+                         g->has_nb[0], g->has_nb[1], chain ? 1 : 0);
+    return;
+  }
   launch_coalesce(g->Q, g->prec, fa, fb, dst, g->dev[L].coal_fill, g->dev[L].coal_cand, H.coal_n[0], H.coal_n[1], mode,
                   g->stream, spin ? g->flags : nullptr, g->has_nb[0], g->has_nb[1], chain ? 1 : 0);
 }
@@ -304,6 +340,7 @@ void update_halo_spin(lbm_grid* g) {
   bool all = true;
   for (int sd = 0; sd < 2; ++sd)
     if (g->has_nb[sd] && !(g->connected[sd] && g->peer_other_gpu[sd])) all = false;
+  g->nb_other_gpu = all;
   if (const char* e = getenv("LBMR_HALO_SPIN")) all = e[0] == '1';
   g->halo_spin = all;
 }
@@ -369,8 +406,13 @@ void launch_F_typed(lbm_grid* g, int L, int64_t k, int kind, cudaEvent_t mid = n
     launch_vavg(g->Q, g->prec, g->dev[L].vavg, (int32_t)(H.vavg.size() / 36), g->dev[L].pop[k & 1],
                 g->dev[L + 1].pop[1], g->dev[L + 1].pop[0], g->bc_dev, g->face_dev, g->dev[L].vtemp, g->stream);
   // coalescence ghosts of C_L^k from C_{L+1}^{2k-1} and C_{L+1}^{2k} (both ready now)
-  if (level_has_coal(g, L)) {
-    if (g->n_ranks > 1 && !g->halo_spin) {
+  if (level_has_coal(g, L) && fused_gather(sched) && !g->host[L].cg_dest.empty()) {
+    // CTA_GATHER: F_L^k's CTAs gather their own cells' links (no launch)
+    p.cg_qoff = g->dev[L].cg_qoff;
+    p.cg_cand = g->dev[L].cg_cand;
+    p.cg_dest = g->dev[L].cg_dest;
+  } else if (level_has_coal(g, L)) {
+    if (g->n_ranks > 1 && !gather_spins(g)) {
       // the gather reads L+1 halo cells: it follows the neighbour wait of F_L^k,
       // which launch_level_step issues first; issue an explicit wait here instead
       launch_halo_wait(p.flags, p.has_nb[0], p.has_nb[1], g->stream);
@@ -668,7 +710,8 @@ static int64_t planned_device_bytes(const std::vector<HostLevel>& host, int Q, s
     t += up(H.blkmap.size(), 4) + up(H.types.size(), 1) + up(H.origin.size(), 4) + up(H.nbr.size(), 4) +
          up(H.special_slot.size(), 4) + up(H.cellinfo.size(), 4) + up(H.bmask.size(), 4) + up(H.links.size(), 4) +
          up(H.coal.size(), 4) + up(H.bpeer.size(), 4) + up(H.ghost_fill.size(), 4) + up(H.coal_fill.size(), 4) +
-         up(H.coal_cand.size(), 4) + up(H.sc_qoff.size(), 4) + up(H.sc_items.size(), 4) + up(H.vfill.size(), 4) +
+         up(H.coal_cand.size(), 4) + up(H.coal_wcand.size(), 4) + up(H.coal_wdst.size(), 4) + up(H.cg_qoff.size(), 4) + up(H.cg_cand.size(), 4) + up(H.cg_dest.size(), 4) +
+         up(H.sc_qoff.size(), 4) + up(H.sc_items.size(), 4) + up(H.vfill.size(), 4) +
          up(H.vavg.size(), 4) + al((H.vavg.size() / 36) * ts) +
          2 * al((size_t)H.nfluid * Q * kCells * ts);
   if (n_ranks > 1) t += al(4 * sizeof(unsigned long long));
@@ -677,7 +720,7 @@ static int64_t planned_device_bytes(const std::vector<HostLevel>& host, int Q, s
 }
 
 static void fill_info(const std::vector<HostLevel>& host, int Q, int prec, int n_ranks, lbm_grid_info* info,
-                      int sched = 0, bool halo_spin = false) {
+                      int sched = 0, bool halo_spin = false, bool gather_spin = false) {
   std::memset(info, 0, sizeof(*info));
   info->levels = (int32_t)host.size();
   info->Q = Q;
@@ -689,8 +732,11 @@ static void fill_info(const std::vector<HostLevel>& host, int Q, int prec, int n
   const bool waits = n_ranks > 1 && !halo_spin;
   if (waits) info->launches_per_step += info->kernels_per_step;
   for (size_t L = 0; L < host.size(); ++L) {
-    // the coalescence gather before every F_L^k (and its own halo wait when partitioned)
-    if (!host[L].coal_fill.empty()) info->launches_per_step += ((int64_t)1 << L) * (waits ? 2 : 1);
+    // the coalescence gather before every F_L^k (and its own halo wait when
+    // partitioned), unless fused into F_L^k (product)
+    const bool gather_waits = n_ranks > 1 && !gather_spin;
+    if (!host[L].coal_fill.empty() && !fused_gather(sched))
+      info->launches_per_step += ((int64_t)1 << L) * (gather_waits ? 2 : 1);
     if (!host[L].vavg.empty()) info->launches_per_step += (int64_t)2 << L;
     // ablation schedules (lbm_set_schedule): split kernels per level-substep
     const int64_t sub = (int64_t)1 << L;
@@ -706,6 +752,8 @@ static void fill_info(const std::vector<HostLevel>& host, int Q, int prec, int n
     info->special_blocks[L] = host[L].nspecial;
     info->special_cells[L] = host[L].special_cells;
     info->total_blocks[L] = host[L].nblocks;
+    info->coal_links[L] = host[L].coal_n[0] + host[L].coal_n[1];
+    info->coal_wide[L] = host[L].coal_n[1];
   }
 }
 
@@ -745,6 +793,7 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
   g->prec = d->precision;
   g->tsize = d->precision == LBM_FP32 ? 4 : 8;
   g->pdl = getenv("LBMR_NO_PDL") == nullptr;
+  if (const char* e = getenv("LBMR_GATHER_WARP")) g->gather_warp = e[0] != '0';
   if (const char* e = getenv("LBMR_PREFETCH")) g->prefetch = std::max(0, atoi(e));
   for (int c = 0; c < 256; ++c) {
     g->bc_host[c].kind = LBM_BC_NOSLIP;
@@ -820,6 +869,11 @@ lbm_status lbm_grid_create(const lbm_grid_desc* d, int32_t levels, const uint8_t
     if ((s = dev_upload(g, &D.ghost_fill, H.ghost_fill))) return cleanup(s);
     if ((s = dev_upload(g, &D.coal_fill, H.coal_fill))) return cleanup(s);
     if ((s = dev_upload(g, &D.coal_cand, H.coal_cand))) return cleanup(s);
+    if ((s = dev_upload(g, &D.coal_wcand, H.coal_wcand))) return cleanup(s);
+    if ((s = dev_upload(g, &D.coal_wdst, H.coal_wdst))) return cleanup(s);
+    if ((s = dev_upload(g, &D.cg_qoff, H.cg_qoff))) return cleanup(s);
+    if ((s = dev_upload(g, &D.cg_cand, H.cg_cand))) return cleanup(s);
+    if ((s = dev_upload(g, &D.cg_dest, H.cg_dest))) return cleanup(s);
     if ((s = dev_upload(g, &D.sc_qoff, H.sc_qoff))) return cleanup(s);
     if ((s = dev_upload(g, &D.sc_items, H.sc_items))) return cleanup(s);
     if ((s = dev_upload(g, &D.vfill, H.vfill))) return cleanup(s);
@@ -1402,7 +1456,7 @@ lbm_status lbm_stats(lbm_grid* g, int64_t* leaves, double* mass) {
 lbm_status lbm_grid_get_info(const lbm_grid* g, lbm_grid_info* info) {
   g_err.clear();
   if (!g || !info) return fail(LBM_E_INVAL, "NULL argument");
-  fill_info(g->host, g->Q, g->prec, g->n_ranks, info, g->sched, g->halo_spin);
+  fill_info(g->host, g->Q, g->prec, g->n_ranks, info, g->sched, g->halo_spin, gather_spins(g));
   info->device_bytes = g->device_bytes;
   info->steps_done = g->steps;
   return LBM_OK;

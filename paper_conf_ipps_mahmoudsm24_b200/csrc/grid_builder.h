@@ -47,6 +47,22 @@ struct HostLevel {
   std::vector<uint32_t> coal_cand;    // SoA fine candidate population indices (level L+1), ~0u = empty:
                                       // [kCoalSlots][coal_n[0]] then [kCoalSlotsMax][coal_n[1]]
   int64_t coal_n[2] = {0, 0};         // entries with |B| <= kCoalSlots, and the others
+  // the same gather list for the warp-cooperative gather kernel: 4-slot units
+  // (array of structures, one 16-byte unit per 4 lanes), the entries with
+  // |B| <= 4 first, then the others as two units each starting at an even
+  // unit (one warp holds both); destination population index per unit (~0u:
+  // second unit of a pair, or padding)
+  std::vector<uint32_t> coal_wcand;   // [nunits][4]
+  std::vector<uint32_t> coal_wdst;    // [nunits]
+  int64_t coal_wpair = 0;             // first unit of the pair segment
+  // Coalescence fused into the coarse level kernel (product schedule,
+  // DESIGN.md §6): per 128-cell quarter block of a launched block, the Eq.11
+  // gathers its own fluid leaves need, as units of 4 candidate slots (an
+  // entry with |B| > 4 takes two consecutive units, the first never the last
+  // of an 8-unit warp group, so one warp holds both)
+  std::vector<uint32_t> cg_qoff;      // [4 nlaunch + 1] CSR offsets into the units
+  std::vector<uint32_t> cg_cand;      // [nunits][4] fine candidate population indices (level L+1), ~0u = empty
+  std::vector<uint32_t> cg_dest;      // [nunits] quarter-local cell | q << 7 | kind << 12 (lattice.h kCg*)
   // atomic form of Accumulate (ablation schedule LBM_SCHED_ATOMIC_A): this
   // level's contributions to the coarser level's coalescence entries,
   // grouped by the 128-cell quarter block of the contributing fine cell

@@ -71,6 +71,13 @@ struct StepParams {
   const uint4* sc_items;        // {fine population index, coarse slot, |B|, 0}
   T* acc;                       // coarse buffer receiving the scatter (C_{L-1}^{ceil((k+1)/2)})
   int32_t sc_scaled;            // 1: add v / (2|B|) (division fused), 0: add v (separate O kernel)
+  // Coalescence fused into this kernel (product schedule):
+  // units of the Eq.11 gathers per 128-cell quarter-block CTA (grid_builder.h
+  // cg_*), summed from fa / fb by warp shuffles into the CTA's shared column;
+  // nullptr: the coalescence ghosts were filled by a gather kernel before
+  const uint32_t* cg_qoff;      // [4 nfluid + 1]
+  const uint32_t* cg_cand;      // [nunits][4]
+  const uint32_t* cg_dest;      // [nunits]
   // 1: launched as the programmatic dependent (PDL) of the coalescence gather
   // that fills this kernel's coalescence ghosts: CTAs of blocks that pull
   // them (record word kRecCoalPull) wait for the gather at their start, all
@@ -113,6 +120,14 @@ void launch_coalesce(int Q, int precision, const void* fa, const void* fb, void*
                      const uint32_t* cand, int64_t n_main, int64_t n_ovf, int mode, cudaStream_t s,
                      const unsigned long long* spin_flags = nullptr, int nb0 = 0, int nb1 = 0,
                      int pdl_chain = 0);
+
+// The same gather, warp-cooperative: 4 lanes per 4-slot unit (grid_builder.h
+// coal_wcand / coal_wdst; units [pair, n) form |B| > 4 pairs), the values
+// added by warp shuffles in the order of launch_coalesce (bitwise equal).
+void launch_coalesce_warp(int precision, const void* fa, const void* fb, void* dst, const uint32_t* cand,
+                          const uint32_t* udst, int64_t n_units, int64_t pair, int mode, cudaStream_t s,
+                          const unsigned long long* spin_flags = nullptr, int nb0 = 0, int nb1 = 0,
+                          int pdl_chain = 0);
 
 // rho / u (double) of n cells given by population cell index block*512+local
 // (-1 -> NaN), read from the post-collision buffer `pop`.

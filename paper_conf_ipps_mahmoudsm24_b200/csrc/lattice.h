@@ -94,6 +94,11 @@ constexpr unsigned kVtNone = 0, kVtA = 1, kVtB = 2, kVtC = 3;
 // link of a planar interface; at most 7 of the 8 candidates 2p - e_q + c lie
 // outside the coarse leaf p (the one inside is ABSENT), so 7 bounds |B|.
 constexpr uint32_t kCoalSlots = 4, kCoalSlotsMax = 7;
+// fused coalescence units (grid_builder.h cg_dest): kind = dest >> 12
+//  kCgSingle  an entry with |B| <= 4 (its 4 slots)
+//  kCgPair    the first unit of an entry with |B| > 4 (slots 0..3; 4..6 in the next unit)
+//  kCgSkip    the second unit of a pair, or padding
+constexpr uint32_t kCgSingle = 0, kCgPair = 1, kCgSkip = 2;
 
 // cell type codes stored per block (mask codes + derived states)
 constexpr unsigned char kAbsent = 0;    // covered by a coarser leaf, or outside the domain

@@ -791,7 +791,81 @@ __device__ __forceinline__ void halo_store(const StepParams<T>& P, const T (&g)[
 template <int Q>
 constexpr bool kEarlyBounce = (Q == 27) || LBMR_EARLY_BOUNCE_Q19;
 
-template <int Q, int COLL, typename T, bool HALO, bool COLLIDE = true, int NT = 256>
+// Coalescence fused into the coarse level kernel (schedule
+// LBM_SCHED_CTA_GATHER): before its cells need them, the CTA evaluates the Eq.11
+// gathers (R-A2/R-A3) of its own fluid leaves' coalescence links,
+// units [a, e) of P.cg_*.  Four lanes per unit: lane m loads candidate slot m
+// of C_{L+1}^{2k-1} (fa) and of C_{L+1}^{2k} (fb); the group's first lane
+// adds the values through __shfl_sync in the oracle's order (fa over the
+// slots, then fb; a |B| > 4 entry spans the next group too), divides by 2|B|
+// and writes the result into the destination cell's column of the shared
+// staging buffer and its direction bit into the cell's mask; the cell takes
+// it after its pulls (coal_merge) like a record value.  Runs at the CTA's
+// start, before the populations are live in registers (no spills), U units
+// per group in flight together.  Same terms in the same order as the gather
+// kernel (coalesce_one): bitwise equal to the gather schedule.
+#ifndef LBMR_CG_UNROLL
+#define LBMR_CG_UNROLL 4
+#endif
+template <typename T, int NT>
+__device__ __forceinline__ void coal_fused(const StepParams<T>& P, uint32_t* cmask, unsigned a, unsigned e) {
+  constexpr unsigned FULL = 0xffffffffu;
+  constexpr int U = LBMR_CG_UNROLL, G = NT / 4;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  T* col = reinterpret_cast<T*>(smem_raw);
+  cmask[threadIdx.x] = 0u;
+  __syncthreads();
+  const int lane = threadIdx.x & 31, gl = lane & ~3, m = lane & 3;
+  for (unsigned base = a; base < e; base += G * U) {  // CTA-uniform trip count
+    uint32_t c[U], d[U];
+#pragma unroll
+    for (int j = 0; j < U; ++j) {
+      const unsigned u = base + (unsigned)(j * G) + (threadIdx.x >> 2);
+      const bool in = u < e;
+      c[j] = in ? __ldg(P.cg_cand + 4 * u + m) : ~0u;
+      d[j] = in ? __ldg(P.cg_dest + u) : (kCgSkip << 12);
+    }
+    T va[U], vb[U];
+#pragma unroll
+    for (int j = 0; j < U; ++j) {
+      va[j] = c[j] != ~0u ? __ldg(P.fa + c[j]) : T(0);
+      vb[j] = c[j] != ~0u ? __ldg(P.fb + c[j]) : T(0);
+    }
+#pragma unroll
+    for (int j = 0; j < U; ++j) {
+      const unsigned kind = d[j] >> 12;
+      const unsigned vm = (__ballot_sync(FULL, c[j] != ~0u) >> gl) & (kind == kCgPair ? 0xffu : 0xfu);
+      T acc = T(0);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        const T v = __shfl_sync(FULL, va[j], gl + i);
+        if ((vm >> i) & 1u) acc += v;
+      }
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        const T v = __shfl_sync(FULL, vb[j], gl + i);
+        if ((vm >> i) & 1u) acc += v;
+      }
+      if (m == 0 && kind != kCgSkip && vm) {
+        const unsigned t = d[j] & 127u, q = (d[j] >> 7) & 31u;
+        col[q * NT + t] = acc / T(2 * __popc(vm));
+        atomicOr(&cmask[t], 1u << q);
+      }
+    }
+  }
+  __syncthreads();
+}
+
+template <int Q, typename T, int NT>
+__device__ __forceinline__ void coal_merge(T (&g)[Q], const uint32_t* cmask) {
+  const uint32_t cm = cmask[threadIdx.x];
+  if (cm) merge_column<Q, T, NT>(g, cm);
+}
+
+// CG: the CTA gathers its cells' coalescence links itself (P.cg_*; level
+// kernels of the CTA_GATHER schedule only: the product's kernels are compiled
+// without this code, so their register assignment is untouched)
+template <int Q, int COLL, typename T, bool HALO, bool COLLIDE = true, int NT = 256, bool CG = false>
 __device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t, bool pdl_gate = false) {
   constexpr unsigned FULL = 0xffffffffu;
   const int lane = threadIdx.x & 31;
@@ -799,6 +873,18 @@ __device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t
   const int rec = __ldg(R + lane);
   const uint32_t fm = (uint32_t)__ldg(R + kRecFluid + (t >> 5));
   const uint32_t sm = (uint32_t)__ldg(R + kRecSpecial + (t >> 5));
+  // fused coalescence: this quarter-block CTA's gather units (CTA-uniform),
+  // evaluated first (one program point for the whole CTA: barriers inside)
+  __shared__ uint32_t cmask[NT];
+  unsigned ca = 0u, ce = 0u;
+  if constexpr (CG && NT == 128) {
+    if (P.cg_qoff) {
+      const unsigned cta = (unsigned)blk * 4u + (unsigned)(t >> 7);
+      ca = __ldg(P.cg_qoff + cta);
+      ce = __ldg(P.cg_qoff + cta + 1);
+      if (ca < ce) coal_fused<T, NT>(P, cmask, ca, ce);
+    }
+  }
   // PDL after the coalescence gather: a warp whose block pulls coalescence
   // ghosts waits for the gather before its pulls (the flag rides in the
   // record the warp has just loaded: no extra round trip)
@@ -811,11 +897,42 @@ __device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t
   // so the plain path keeps its own spill-free register assignment
   constexpr bool kShared = (COLL == LBM_KBC);
 #ifdef LBMR_DEBUG_ALLPLAIN
-  if (true) {  // timing experiment only (wrong results): every warp takes the plain path
+  const bool plain = true;  // timing experiment only (wrong results): every warp takes the plain path
 #else
-  if (fm == FULL && sm == 0u) {
+  const bool plain = (fm == FULL && sm == 0u);  // warp-uniform
 #endif
+  int slot = 0;
+  bool fluid = true, special = false;
+  uint32_t bm = 0u;
+  uint4 ci = make_uint4(0u, 0u, 0u, kNoBCSource);
+  uint32_t cm = 0u;  // coalescence links of the cell (special path)
+  if (plain) {
     pull_all<Q, T, false>(g, P.src, G, rec, blk, true, std::make_integer_sequence<int, Q>{});
+    // the cell's coalescence links from the column (merged in each path:
+    // a common merge point would join the plain path's register assignment
+    // with the special path's)
+    if (CG && ca < ce) coal_merge<Q, T, NT>(g, cmask);
+  } else {
+    slot = __shfl_sync(FULL, rec, kRecSlot);
+    fluid = (fm >> lane) & 1u;
+    special = (sm >> lane) & 1u;
+    if constexpr (kEarlyBounce<Q>) {
+      // bounce-back sources (the cell's own opposite populations) of every
+      // direction some cell of this warp bounces: copied into the thread's
+      // shared-memory column right after the pulls, not after the cell's
+      // info arrives (partly fluid warps without special cells skip the
+      // load: sm is warp-uniform)
+      bm = (sm != 0u && fluid) ? __ldg(P.bmask + (unsigned)slot * kBounceWords + (t >> 5)) : 0u;
+    } else {
+      // the cell's info first, its bounce copies once it has arrived
+      if (special) ci = __ldg(P.cellinfo + (unsigned)slot * kCells + t);
+    }
+    pull_all<Q, T, true>(g, P.src, G, rec, blk, fluid, std::make_integer_sequence<int, Q>{});
+    // the cell's coalescence links join its record merge below (never
+    // bounce or record links; the warp-union bounce copies skip them)
+    if (CG && ca < ce) cm = cmask[threadIdx.x];
+  }
+  if (plain) {
     if (!kShared) {
       if (COLLIDE) collide<Q, COLL, T>(g, P.omega);
       store_cell<Q, T>(g, P.dst, blk, t);
@@ -823,35 +940,20 @@ __device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t
       return;
     }
   } else {
-    const int slot = __shfl_sync(FULL, rec, kRecSlot);
-    const bool fluid = (fm >> lane) & 1u;
-    const bool special = (sm >> lane) & 1u;
     if constexpr (kEarlyBounce<Q>) {
-      // bounce-back sources (the cell's own opposite populations) of every
-      // direction some cell of this warp bounces: copied into the thread's
-      // shared-memory column right after the pulls, not after the cell's
-      // info arrives (partly fluid warps without special cells skip the
-      // load: sm is warp-uniform)
-      const uint32_t bm = (sm != 0u && fluid) ? __ldg(P.bmask + (unsigned)slot * kBounceWords + (t >> 5)) : 0u;
-      pull_all<Q, T, true>(g, P.src, G, rec, blk, fluid, std::make_integer_sequence<int, Q>{});
 #ifndef LBMR_DEBUG_NOSLOW
-      if (bm) bounce_issue<Q, T, NT>(P, bm, own);
+      if (bm & ~cm) bounce_issue<Q, T, NT>(P, bm & ~cm, own);
 #endif
       if (!fluid) return;
-      uint4 ci = make_uint4(0u, 0u, 0u, kNoBCSource);
       if (special) ci = __ldg(P.cellinfo + (unsigned)slot * kCells + t);
 #ifndef LBMR_DEBUG_NOSLOW
-      if (bm) asm volatile("cp.async.wait_all;" ::: "memory");
+      if (bm & ~cm) asm volatile("cp.async.wait_all;" ::: "memory");
       const uint32_t recs = ci.x & ((1u << Q) - 1u);
       if (recs) resolve_slow_links<Q, T, NT>(P, recs, ci.y, blk, t);  // into the column, disjoint from ci.z
-      if (ci.z | recs) merge_column<Q, T, NT>(g, ci.z | recs);
+      if (ci.z | recs | cm) merge_column<Q, T, NT>(g, ci.z | recs | cm);
       if (ci.z) bounce_fix<Q, T>(P, g, ci.z, ci.w);
 #endif
     } else {
-      // the cell's info first, its bounce copies once it has arrived
-      uint4 ci = make_uint4(0u, 0u, 0u, kNoBCSource);
-      if (special) ci = __ldg(P.cellinfo + (unsigned)slot * kCells + t);
-      pull_all<Q, T, true>(g, P.src, G, rec, blk, fluid, std::make_integer_sequence<int, Q>{});
       if (!fluid) return;
 #ifndef LBMR_DEBUG_NOSLOW
       if (ci.z) {
@@ -861,9 +963,9 @@ __device__ __forceinline__ void step_cell(const StepParams<T>& P, int blk, int t
         bounce_fix<Q, T>(P, g, ci.z, ci.w);
       }
       const uint32_t recs = ci.x & ((1u << Q) - 1u);
-      if (recs) {
-        resolve_slow_links<Q, T, NT>(P, recs, ci.y, blk, t);
-        merge_column<Q, T, NT>(g, recs);
+      if (recs | cm) {
+        if (recs) resolve_slow_links<Q, T, NT>(P, recs, ci.y, blk, t);
+        merge_column<Q, T, NT>(g, recs | cm);
       }
 #endif
     }
@@ -935,7 +1037,7 @@ __device__ __forceinline__ void prefetch_block(const StepParams<T>& P, int blk) 
 __device__ __forceinline__ void pdl_wait() { griddep_wait(); }
 __device__ __forceinline__ void pdl_launch_dependents() { asm volatile("griddepcontrol.launch_dependents;" :::); }
 
-template <int Q, int COLL, typename T>
+template <int Q, int COLL, typename T, bool CG = false>
 __global__ void __launch_bounds__(StepCta<Q, COLL, T>::threads, StepCta<Q, COLL, T>::min_blocks)
     level_step_all(const StepParams<T> P) {
   constexpr int NT = StepCta<Q, COLL, T>::threads, PB = StepCta<Q, COLL, T>::per_block;
@@ -959,7 +1061,7 @@ __global__ void __launch_bounds__(StepCta<Q, COLL, T>::threads, StepCta<Q, COLL,
   // under PDL the gather may still be running: warps whose block pulls a
   // coalescence ghost wait for it before their pulls (inside step_cell), all
   // others after their work (a second wait returns at once)
-  step_cell<Q, COLL, T, false, true, NT>(P, b / PB, (b % PB) * NT + threadIdx.x, P.pdl != 0);
+  step_cell<Q, COLL, T, false, true, NT, CG>(P, b / PB, (b % PB) * NT + threadIdx.x, P.pdl != 0);
   if (P.sc_qoff) accumulate_scatter<T, NT>(P, b / PB, (b % PB) * NT);
   if (P.pdl) pdl_wait();
 }
@@ -1237,6 +1339,49 @@ __global__ void __launch_bounds__(256) coalesce_kernel(const T* __restrict__ fa,
   }
 }
 
+// Warp-cooperative form of the gather (launch_coalesce_warp): four lanes per
+// 4-slot unit, lane m loading candidate slot m of fa and fb (one coalesced
+// 16-byte unit load per four lanes); the unit's first lane adds the values
+// through __shfl_sync in the oracle's order (fa slots then fb slots; a pair
+// spans the next unit too), like coalesce_one.
+template <typename T>
+__global__ void __launch_bounds__(256) coalesce_warp_kernel(const T* __restrict__ fa, const T* __restrict__ fb,
+                                                            T* dst, const uint32_t* __restrict__ cand,
+                                                            const uint32_t* __restrict__ udst, int64_t n, int64_t pair,
+                                                            int mode, const unsigned long long* spin_flags, int nb0,
+                                                            int nb1, int pdl_chain) {
+  constexpr unsigned FULL = 0xffffffffu;
+  if (pdl_chain) pdl_wait();
+  pdl_launch_dependents();
+  if (spin_flags) halo_spin_cta(spin_flags, nb0, nb1);
+  const int64_t u = (int64_t)blockIdx.x * 64 + (threadIdx.x >> 2);
+  const int lane = threadIdx.x & 31, gl = lane & ~3, m = lane & 3;
+  const bool in = u < n;
+  const uint32_t c = in ? __ldg(cand + 4 * u + m) : ~0u;
+  uint32_t d = ~0u;
+  if (in && m == 0) d = __ldg(udst + u);
+  const T va = (fa && c != ~0u) ? __ldg(fa + c) : T(0);
+  const T vb = (fb && c != ~0u) ? __ldg(fb + c) : T(0);
+  const T v0 = (in && m == 0 && d != ~0u && (mode & kCoalFromDst)) ? dst[d] : T(0);
+  const unsigned vm = (__ballot_sync(FULL, c != ~0u) >> gl) & (u >= pair ? 0xffu : 0xfu);
+  T acc = v0;
+  if (fa) {
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const T v = __shfl_sync(FULL, va, gl + i);
+      if ((vm >> i) & 1u) acc += v;
+    }
+  }
+  if (fb) {
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const T v = __shfl_sync(FULL, vb, gl + i);
+      if ((vm >> i) & 1u) acc += v;
+    }
+  }
+  if (m == 0 && d != ~0u) dst[d] = (mode & kCoalDivide) ? acc / T(2 * __popc(vm)) : acc;
+}
+
 template <int Q, typename T>
 __global__ void __launch_bounds__(256) vavg_gather(const uint32_t* __restrict__ ent, int n, const T* A, const T* B,
                                                    const T* C, const BCEntry* bc, const uint8_t* face_cls, T* tmp) {
@@ -1335,6 +1480,20 @@ void launch_coalesce(int Q, int precision, const void* fa, const void* fb, void*
                      pdl_chain);
 }
 
+void launch_coalesce_warp(int precision, const void* fa, const void* fb, void* dst, const uint32_t* cand,
+                          const uint32_t* udst, int64_t n_units, int64_t pair, int mode, cudaStream_t s,
+                          const unsigned long long* spin_flags, int nb0, int nb1, int pdl_chain) {
+  if (n_units <= 0) return;
+  const unsigned grid = (unsigned)((n_units + 63) / 64);
+  if (precision == LBM_FP32)
+    launch_maybe_pdl(pdl_chain != 0, coalesce_warp_kernel<float>, dim3(grid), dim3(256), 0, s, (const float*)fa,
+                     (const float*)fb, (float*)dst, cand, udst, n_units, pair, mode, spin_flags, nb0, nb1, pdl_chain);
+  else
+    launch_maybe_pdl(pdl_chain != 0, coalesce_warp_kernel<double>, dim3(grid), dim3(256), 0, s, (const double*)fa,
+                     (const double*)fb, (double*)dst, cand, udst, n_units, pair, mode, spin_flags, nb0, nb1,
+                     pdl_chain);
+}
+
 // ---------------------------------------------------------------- dispatch
 // dynamic shared memory of the stepping kernels: the slow-link staging
 // buffer sv[Q][256] of resolve_slow
@@ -1371,7 +1530,8 @@ static void launch_typed(int kind, const void* params, cudaStream_t s) {
     const int gct = (trail_count(p) + NT - 1) / NT;
     const dim3 grid(p.nfluid * StepCta<Q, COLL, T>::per_block + gct), blk(NT);
     const size_t smem = (size_t)Q * NT * sizeof(T);
-    launch_maybe_pdl(p.pdl || p.pdl_chain, level_step_all<Q, COLL, T>, grid, blk, smem, s, p);
+    if (p.cg_qoff) launch_maybe_pdl(p.pdl || p.pdl_chain, level_step_all<Q, COLL, T, true>, grid, blk, smem, s, p);
+    else launch_maybe_pdl(p.pdl || p.pdl_chain, level_step_all<Q, COLL, T>, grid, blk, smem, s, p);
   }
 }
 
@@ -1383,6 +1543,8 @@ template <int Q, int COLL, typename T>
 static void preload_variant() {
   cudaFuncSetAttribute(level_step_all<Q, COLL, T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                        (int)slow_smem<Q, T>());
+  cudaFuncSetAttribute(level_step_all<Q, COLL, T, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                       (int)slow_smem<Q, T>());
   cudaFuncSetAttribute(level_step_halo<Q, COLL, T, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                        (int)slow_smem<Q, T>());
   cudaFuncSetAttribute(level_stream<Q, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)slow_smem<Q, T>());
@@ -1390,6 +1552,7 @@ static void preload_variant() {
   cudaFuncGetAttributes(&a, level_stream<Q, T>);
   cudaFuncGetAttributes(&a, level_collide_inplace<Q, COLL, T>);
   cudaFuncGetAttributes(&a, level_step_all<Q, COLL, T>);
+  cudaFuncGetAttributes(&a, level_step_all<Q, COLL, T, true>);
   cudaFuncGetAttributes(&a, level_collide<Q, COLL, T>);
   cudaFuncGetAttributes(&a, level_step_halo<Q, COLL, T, true>);
   cudaFuncGetAttributes(&a, level_step_halo<Q, COLL, T, false>);
@@ -1419,6 +1582,8 @@ void preload_kernels() {
   cudaFuncGetAttributes(&a, probe_kernel<19, double>);
   cudaFuncGetAttributes(&a, probe_kernel<27, double>);
   cudaFuncGetAttributes(&a, coalesce_kernel<double>);
+  cudaFuncGetAttributes(&a, coalesce_warp_kernel<float>);
+  cudaFuncGetAttributes(&a, coalesce_warp_kernel<double>);
   cudaFuncGetAttributes(&a, init_eq_kernel<19, float>);
   cudaFuncGetAttributes(&a, init_eq_kernel<27, float>);
   cudaFuncGetAttributes(&a, init_eq_kernel<19, double>);

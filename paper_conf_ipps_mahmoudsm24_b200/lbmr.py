@@ -24,6 +24,7 @@ FP32, FP64 = 0, 1
 BC_NOSLIP, BC_VELOCITY, BC_OUTFLOW = 0, 1, 2
 SCHED_FUSED, SCHED_UNFUSED, SCHED_NO_GRAPH = 0, 1, 2
 SCHED_SPLIT_E, SCHED_SPLIT_A, SCHED_ATOMIC_A, SCHED_SPLIT_O = 4, 8, 16, 32
+SCHED_CTA_GATHER = 64
 # the paper's Fig. 4 configurations as schedule bit sets
 FIG4 = {
     "4b": SCHED_UNFUSED | SCHED_SPLIT_E | SCHED_SPLIT_A | SCHED_SPLIT_O,  # modified baseline: C, A, S, E, O
@@ -31,7 +32,8 @@ FIG4 = {
     "4d": SCHED_UNFUSED | SCHED_SPLIT_A | SCHED_SPLIT_O,  # SE fused
     "4e": SCHED_UNFUSED | SCHED_ATOMIC_A,  # CA, SE and SO fused
     "4f": SCHED_ATOMIC_A,  # CASE and SO fused (the paper's design)
-    "product": SCHED_FUSED,  # fused level kernels, gather A+A+O (deterministic)
+    "product": SCHED_FUSED,  # fused level kernels, warp-cooperative A+A+O gather kernel (deterministic)
+    "cta_gather": SCHED_CTA_GATHER,  # A+A+O gathered inside F_L^k by each CTA (no gather kernel)
 }
 VARIANT_PAPER, VARIANT_VOLUMETRIC = 0, 1
 
@@ -65,6 +67,7 @@ class GridInfo(ctypes.Structure):
         ("device_bytes", ctypes.c_int64), ("steps_done", ctypes.c_int64),
         ("launches_per_step", ctypes.c_int64),
         ("block_offset", (ctypes.c_int32 * 3) * 16),
+        ("coal_links", ctypes.c_int64 * 16), ("coal_wide", ctypes.c_int64 * 16),
     ]
 
 

@@ -86,7 +86,7 @@ def test_schedule_switch_mid_run():
 def test_bad_schedule_mode():
     lbmr = _lbmr()
     g = lbmr.grid_from_problem(I.cavity2(), precision=FP32)
-    for bad in (64, -1, lbmr.SCHED_SPLIT_A | lbmr.SCHED_ATOMIC_A):
+    for bad in (128, -1, lbmr.SCHED_SPLIT_A | lbmr.SCHED_ATOMIC_A):
         with pytest.raises(lbmr.LBMError):
             g.set_schedule(bad)
     g.close()
