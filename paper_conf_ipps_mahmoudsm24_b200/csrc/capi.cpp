@@ -106,7 +106,9 @@ struct lbm_grid {
   int sched = LBM_SCHED_FUSED;  // lbm_set_schedule
   bool pdl = true;              // programmatic dependent launch of F_L^k after its gather (LBMR_NO_PDL=1: off)
   bool gather_warp = false;      // warp-cooperative gather kernel (LBMR_GATHER_WARP=1; default thread per entry)
-  int32_t prefetch = 16;        // L2 prefetch distance of the level kernels, in blocks (LBMR_PREFETCH; 0: off)
+  // L2 prefetch distance of the level kernels, in blocks (LBMR_PREFETCH; 0: off); re-swept
+  // (profiles/r02_prefetch_resweep.txt): 64 vs 16 cfg5 fp32 +0.6 %, cfg4 KBC +0.4 %, Tab. I s3 +0.3 %
+  int32_t prefetch = 64;
   bool peer_other_gpu[2] = {false, false};  // the connected neighbour on this side is on another GPU
   bool halo_spin = false;       // in-kernel halo waits (every connected neighbour on another GPU)
   bool nb_other_gpu = false;    // every connected neighbour is on another GPU (halo_spin without the env override)
