@@ -21,3 +21,9 @@ ncu --set full --clock-control none --import-source on -k regex:level_step_all -
     python bench.py --traffic-child --config uniform512 --precision fp32 > /dev/null 2>&1
 bash tools/gpu_sweep.sh ${tag}sweep > gpurun_out/${tag}_sweep_table.txt 2>&1
 cat gpurun_out/${tag}_sweep_table.txt
+# summaries on the box (gpurun copies back at most 64 MiB): text summaries of every report, then the reports go
+python tools/launch_summary.py gpurun_out/${tag}_launches.csv > gpurun_out/${tag}_launches_summary.txt 2>&1
+for r in gpurun_out/${tag}_prof*.ncu-rep; do echo "# $r"; python tools/ncu_summary.py $r; done > gpurun_out/${tag}_ncu_summary.txt 2>&1
+ncu -i gpurun_out/${tag}_prof.ncu-rep --page source --csv --print-source sass > gpurun_out/${tag}_ncu_source_cfg5.csv 2>/dev/null
+gzip -f gpurun_out/${tag}_ncu_source_cfg5.csv
+rm -f gpurun_out/${tag}_prof*.ncu-rep
