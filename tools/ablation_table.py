@@ -9,10 +9,11 @@ import json
 import os
 import sys
 
-ORDER = ["fig4b", "fig4c", "fig4d", "fig4e", "fig4f", "unfused", "fused"]
+ORDER = ["fig4b", "fig4c", "fig4d", "fig4e", "fig4f", "unfused", "cta_gather", "fused"]
 LABEL = {"fig4b": "4b modified baseline (C, A, S, E, O separate)", "fig4c": "4c CA fused (atomic Accumulate)",
          "fig4d": "4d SE fused", "fig4e": "4e CA, SE, SO fused", "fig4f": "4f CASE + SO fused (atomic A)",
-         "unfused": "C | SEO (gather A+A+O)", "fused": "product: CSEO fused, gather A+A+O (PDL)"}
+         "unfused": "C | SEO (gather A+A+O)", "cta_gather": "CSEO + A+A+O in one kernel (in-CTA gather)",
+         "fused": "product: CSEO fused, gather A+A+O (PDL)"}
 
 
 def main(prefix):
