@@ -206,7 +206,9 @@ template <typename T, typename Acc>
 __device__ __forceinline__ void collide_kbc_acc(Acc& acc, T omega) {
   constexpr int Q = 27;
   T drho = acc.get(0), jx = T(0), jy = T(0), jz = T(0);
-  T sxx = T(0), syy = T(0), szz = T(0), sxy = T(0), sxz = T(0), syz = T(0);
+  // S_xx - S_zz and S_yy - S_zz accumulated directly: a pair with both (or
+  // neither) of e_x, e_z nonzero adds nothing to S_xx - S_zz
+  T dxz = T(0), dyz = T(0), sxy = T(0), sxz = T(0), syz = T(0);
 #pragma unroll
   for (int q = 1; q < Q; q += 2) {
     const T gq = acc.get(q), gq1 = acc.get(q + 1);
@@ -216,17 +218,16 @@ __device__ __forceinline__ void collide_kbc_acc(Acc& acc, T omega) {
     if (ex(q) > 0) jx += df; else if (ex(q) < 0) jx -= df;
     if (ey(q) > 0) jy += df; else if (ey(q) < 0) jy -= df;
     if (ez(q) > 0) jz += df; else if (ez(q) < 0) jz -= df;
-    if (ex(q)) sxx += sm;
-    if (ey(q)) syy += sm;
-    if (ez(q)) szz += sm;
+    if (ex(q) && !ez(q)) dxz += sm; else if (!ex(q) && ez(q)) dxz -= sm;
+    if (ey(q) && !ez(q)) dyz += sm; else if (!ey(q) && ez(q)) dyz -= sm;
     if (ex(q) * ey(q) > 0) sxy += sm; else if (ex(q) * ey(q) < 0) sxy -= sm;
     if (ex(q) * ez(q) > 0) sxz += sm; else if (ex(q) * ez(q) < 0) sxz -= sm;
     if (ey(q) * ez(q) > 0) syz += sm; else if (ey(q) * ez(q) < 0) syz -= sm;
   }
   const T inv = recip<T>(T(1) + drho);
   const T jxi = jx * inv, jyi = jy * inv, jzi = jz * inv;
-  const T nxz = (sxx - szz) - (jx * jxi - jz * jzi);
-  const T nyz = (syy - szz) - (jy * jyi - jz * jzi);
+  const T nxz = dxz - (jx * jxi - jz * jzi);
+  const T nyz = dyz - (jy * jyi - jz * jzi);
   const T sixth = T(1) / T(6);
   const T sx = (T(2) * nxz - nyz) * sixth, sy = (T(2) * nyz - nxz) * sixth, sz = -(nxz + nyz) * sixth;
   const T exy = (sxy - jx * jyi) * T(0.25), exz = (sxz - jx * jzi) * T(0.25), eyz = (syz - jy * jzi) * T(0.25);
@@ -274,12 +275,20 @@ __device__ __forceinline__ void collide_kbc_acc(Acc& acc, T omega) {
         i0 = (a - asym) * r;
         i1 = (a + asym) * r;
       }
-      const T s0 = ds(q), s1 = ds(q + 1);
-      const T h0 = (acc.get(q) - (sym + asym)) - s0, h1 = (acc.get(q + 1) - (sym - asym)) - s1;
-      sh += s0 * h0 * i0;
-      hh += h0 * h0 * i0;
-      sh2 += s1 * h1 * i1;
-      hh2 += h1 * h1 * i1;
+      // Δs is even in e (ds(q) == ds(q + 1)) and zero on the corner
+      // directions: h = (g - (g^eq_sym + Δs)) ∓ g^eq_asym, and the <Δs|Δh>
+      // terms of the corners are skipped (compile time)
+      const bool kHasS = ex(q) * ex(q) + ey(q) * ey(q) + ez(q) * ez(q) < 3;
+      const T sq = ds(q);
+      const T u = kHasS ? sym + sq : sym;
+      const T h0 = (acc.get(q) - u) - asym, h1 = (acc.get(q + 1) - u) + asym;
+      const T t0 = h0 * i0, t1 = h1 * i1;
+      if (kHasS) {
+        sh += sq * t0;
+        sh2 += sq * t1;
+      }
+      hh += h0 * t0;
+      hh2 += h1 * t1;
     }
   }
   sh += sh2;
