@@ -342,6 +342,9 @@ void update_halo_spin(lbm_grid* g) {
   bool all = true;
   for (int sd = 0; sd < 2; ++sd)
     if (g->has_nb[sd] && !(g->connected[sd] && g->peer_other_gpu[sd])) all = false;
+  // test hook: neighbours on SM-disjoint green contexts of one GPU behave like
+  // neighbours on other GPUs (tests/test_gpu_green_partition.py)
+  if (const char* e = getenv("LBMR_TEST_OTHER_GPU")) all = e[0] == '1';
   g->nb_other_gpu = all;
   if (const char* e = getenv("LBMR_HALO_SPIN")) all = e[0] == '1';
   g->halo_spin = all;
