@@ -182,10 +182,12 @@ lbm_status lbm_profile_levels(lbm_grid* g, int32_t n_coarse, double* ms_per_leve
  * accumulated values), §IV and Fig. 4.
  *  LBM_SCHED_FUSED     (0) one fused kernel F_L^k per level-substep (S + E +
  *                      O + BC + C), 2Q values moved per leaf, and one small
- *                      warp-cooperative gather kernel before it doing A + A +
- *                      O from the two retained fine buffers (deterministic,
- *                      warp shuffles; F_L^k its programmatic dependent) — the
- *                      product.
+ *                      gather kernel before it doing A + A + O from the two
+ *                      retained fine buffers (deterministic, one thread per
+ *                      link; F_L^k its programmatic dependent) — the product.
+ *                      (LBMR_GATHER_WARP=1 in the environment at grid creation
+ *                      selects a warp-cooperative form of the same gather:
+ *                      bitwise equal, measured slower.)
  *  LBM_SCHED_UNFUSED   (1) C and S separate: a stream-only kernel S_L^k then
  *                      an in-place collision C_L^{k+1} (4Q values per leaf).
  *  LBM_SCHED_NO_GRAPH  (2) launch the kernels one by one instead of replaying
