@@ -750,9 +750,12 @@ __device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long
 
 template <typename T>
 __device__ __forceinline__ void halo_signal(const StepParams<T>& P, int nproto) {
-  __threadfence_system();
+  // the barrier orders every thread's halo stores before thread 0's
+  // system-scope fence (fences are cumulative), which orders them before the
+  // count: one fence per CTA instead of one per thread
   __syncthreads();
   if (threadIdx.x == 0) {
+    __threadfence_system();
     if (atomicAdd(P.flags + 3, 1ull) == (unsigned long long)(nproto - 1)) {
       P.flags[3] = 0ull;
       P.flags[2] += 1ull;
@@ -1130,27 +1133,35 @@ template <int Q, int COLL, typename T, bool STREAM>
 __global__ void __launch_bounds__(kHaloCtaThreads, (PlainOcc<Q, T, COLL>::value * 256) / kHaloCtaThreads)
     level_step_halo(const StepParams<T> P) {
   constexpr int NT = kHaloCtaThreads, PB = kHaloCtasPerBlock;
-  const int blk = (int)blockIdx.x / PB;
-  const int t = ((int)blockIdx.x % PB) * NT + threadIdx.x;
-  const int main = PB * max(P.nfluid, 1);
+  // CTA order: the cut-plane CTAs [0, nbctas) (blocks stored first), then the
+  // ghost-refresh CTAs, then the interior CTAs.  Both protocol groups sit at
+  // the front, so the completion signal (their last CTA) fires early in the
+  // kernel and a neighbour's next kernel waits for this kernel's cut-plane
+  // part only, not for its end (ranks stay loosely coupled: one kernel of
+  // slack instead of lockstep).
+  const int nfill = halo_fill_ctas(trail_count(P));
+  const int bid = (int)blockIdx.x;
+  const bool fill = bid >= P.nbctas && bid < P.nbctas + nfill;
+  const int mb = bid < P.nbctas ? bid : bid - nfill;  // main CTA index (interior CTAs after the fills)
+  const int blk = mb / PB;
+  const int t = (mb % PB) * NT + threadIdx.x;
   // the wait happened in halo_wait_kernel just before this launch; cut-plane
   // CTAs (which write the neighbour's halo) and ghost-refresh CTAs (which may
   // read L-1 halo cells) count towards this kernel's completion signal
-  const bool fill = (int)blockIdx.x >= main;
-  const bool proto = (int)blockIdx.x < P.nbctas || fill;
+  const bool proto = bid < P.nbctas || fill;
   if (P.pdl_chain) {  // PDL chain: resident during the previous kernel's tail (see level_step_all)
     pdl_wait();
     pdl_launch_dependents();
   }
   if (P.halo_spin && proto) halo_spin_cta(P.flags, P.has_nb[0], P.has_nb[1]);
-  if (!fill && ((int)blockIdx.x % PB) == 0) prefetch_block<Q, T>(P, blk);
+  if (!fill && (mb % PB) == 0) prefetch_block<Q, T>(P, blk);
   if (fill) {
-    trail_fill<Q, T>(P, ((int)blockIdx.x - main) * NT + threadIdx.x);
+    trail_fill<Q, T>(P, (bid - P.nbctas) * NT + threadIdx.x);
   } else if (blk < P.nfluid) {
     if (STREAM) step_cell<Q, COLL, T, true, true, NT>(P, blk, t);
     else collide_cell<Q, COLL, T, true>(P, blk, t);
   }
-  if (proto) halo_signal<T>(P, P.nbctas + halo_fill_ctas(trail_count(P)));
+  if (proto) halo_signal<T>(P, P.nbctas + nfill);
 }
 
 template <int Q, int COLL, typename T>
