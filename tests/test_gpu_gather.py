@@ -113,3 +113,22 @@ def test_partitioned_warp_gather_equals_thread_gather(name, P, monkeypatch):
     a = run()
     monkeypatch.setenv("LBMR_GATHER_WARP", "1")
     _same(a, run())
+
+
+@pytest.mark.parametrize("name", ["cavity2r", "random4", "tunnel_s5"])
+def test_multi_step_graphs_bitwise(name, monkeypatch):
+    """lbm_step(n) replays graphs of several coarse steps when n allows
+    (LBMR_GRAPH_STEPS, default 4) and single-step graphs for the rest: any
+    chunking equals one-step graphs bitwise."""
+    lbmr = _lbmr()
+    prob = PROBLEMS[name]()
+    monkeypatch.setenv("LBMR_GRAPH_STEPS", "1")
+    ref, _ = _run(prob, FP64, 11)
+    for gs, chunks in (("4", (11,)), ("4", (3, 5, 1, 2)), ("3", (7, 4)), ("2", (1, 10))):
+        monkeypatch.setenv("LBMR_GRAPH_STEPS", gs)
+        g = lbmr.grid_from_problem(prob, precision=FP64)
+        for c in chunks:
+            g.step(c)
+        got = [g.macroscopic(L) for L in range(prob.levels)]
+        g.close()
+        _same(got, ref)
